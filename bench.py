@@ -1,0 +1,368 @@
+#!/usr/bin/env python
+"""nu-LPA benchmark (BASELINE.json metric: edges/s = |E| / runtime).
+
+One step = one complete nu-LPA run (Algorithm 1: reset labels, sweeps with
+Pick-Less every 4 iterations until dN/N < tau or 20 iterations) over the
+graph, inputs resident in HBM.  Default workload: the synthetic web-like
+power-law graph of BASELINE.json configs[4] (~40M vertices / 2.2B CSR
+entries, it-2004-shaped, edge weights stored as float32 ones like the
+paper's "weighted, with a default weight of 1" graphs).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+N > 1: launched by torchrun, one rank per GPU; the vertex range is split by
+edge count and labels are exchanged after every sweep (see
+paper_conf_ipps_sahunk25_b200/distributed.py).  Rank 0 prints one JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "edges/s (|E|/runtime)"
+BINS = ("thread", "warp", "block", "giant")
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="web_40m_2200m")
+    ap.add_argument("--weights", choices=["ones", "random", "none"], default="ones",
+                    help="ones: float32 array of 1.0 (the paper's default weight); none: unit-weight fast path")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--scale", type=float, default=1.0, help="shrink the workload (debug only; invalid as a bench number)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=4_000_000, help="vertices of the oracle's web-graph sample")
+    ap.add_argument("--extra", action="store_true", help="also time the unit-weight fast path and sync mode")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------------
+def make_graph(args, device):
+    import synth
+    kw = {}
+    if args.scale != 1.0:
+        base = synth.CONFIGS[args.config]["kw"]
+        if "n" in base:
+            kw["n"] = int(base["n"] * args.scale)
+        if "scale" in base:
+            kw["scale"] = max(10, int(round(base["scale"] + __import__("math").log2(args.scale))))
+        if "R" in base:
+            kw["R"] = int(base["R"] * args.scale ** 0.5)
+    g = synth.make(args.config, device=device, seed=args.seed, weighted=(args.weights == "random"), **kw)
+    return g
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def algorithmic_bytes(st, b, weighted):
+    """Compulsory DRAM bytes of bin b over a run (DESIGN.md 'Kernels and
+    their rooflines'): per processed vertex 4 (bin list) + 16 (two offsets)
+    + 2 (flag read + clear) + 4 (own label); per scanned CSR entry 4 (index)
+    + 4 (weight, if stored); per changed vertex 4 (label write) and per CSR
+    entry of a changed vertex 4 (index re-read) + 1 (neighbour flag write).
+    Neighbour-label gathers are NOT counted (the label array is re-used
+    from cache); this is a lower bound on DRAM traffic."""
+    v = st["vertices_processed"][b]
+    e = st["edges_scanned"][b]
+    c = st["vertices_changed"][b]
+    ce = st["changed_edges"][b]
+    return v * 26 + e * (8 if weighted else 4) + c * 4 + ce * 5
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index=0):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.gpu = gpu_index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = [r.split(", ") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm = [float(r[1]) for r in rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            if len(r) >= 9:
+                for k, nm in enumerate(names):
+                    if r[5 + k].strip() == "Active":
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+# ---------------------------------------------------------------------------
+def cpu_baseline(args):
+    """The oracle (oracle/, plain single-threaded C) on a bounded sample of the
+    same workload family, timed on this host's cores."""
+    import torch
+    import oracle
+    import synth
+    n = args.cpu_sample
+    if args.config.startswith("web"):
+        dev = "cuda" if torch.cuda.is_available() else "cpu"
+        g = synth.web(n=n, seed=args.seed + 1, device=dev).to("cpu")
+        sample = f"synth.web(n={n}) web-like graph, {g.M} CSR entries (same generator as the workload)"
+    else:
+        g = make_graph(args, "cpu")
+        sample = f"the full {args.config} workload"
+    h = oracle.CSR.from_graph(g)
+    if args.weights == "ones":
+        import numpy as np
+        h = oracle.CSR(h.offsets, h.indices, np.ones(h.M, dtype=np.float32))
+    t0 = time.perf_counter()
+    C, it, dn = oracle.lpa(h)
+    dt = time.perf_counter() - t0
+    q = oracle.modularity(h, C)
+    return {"value": h.M / dt, "unit": "edges/s", "cores": 1, "kind": "oracle",
+            "sample": sample + f"; full async oracle run, {it} iterations, {dt:.2f} s, modularity {q:.4f}",
+            "seconds": dt, "iterations": it, "modularity": q, "M": h.M}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cb = cpu_baseline(args)
+    line = {"impl": "reference", "metric": METRIC, "value": cb["value"], "unit": "edges/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": cb["seconds"] * 1e3, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": args.config, "sample": cb["sample"]},
+            "cpu_baseline": {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")},
+            "e2e": {"value": cb["value"], "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------------------
+def run_ours(args):
+    import torch
+    import paper_conf_ipps_sahunk25_b200 as nl
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            raise SystemExit("--gpus N > 1 must be launched with torchrun (one rank per GPU)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        return run_distributed(args, rank, world, local)
+
+    t_gen = time.perf_counter()
+    g = make_graph(args, "cuda")
+    weights = None
+    if args.weights == "ones":
+        weights = torch.ones(g.M, dtype=torch.float32, device="cuda")
+    elif args.weights == "random":
+        weights = g.weights
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - t_gen
+    N, M = g.N, g.M
+    weighted = weights is not None
+    stream = torch.cuda.current_stream()
+    gg = nl.Graph(g.offsets, g.indices, weights)
+    params = dict(timing=1)
+    for _ in range(args.warmup):
+        gg.run(**params)
+    torch.cuda.synchronize()
+    clocks = Clocks(local)
+    clocks.start()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    stats = []
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        stats.append(gg.run(**params))
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    value = M / (ms / 1e3)
+    q = gg.modularity()
+    launches = sum(sum(s["launches"]) + s["other_launches"] for s in stats)
+
+    # roofline of the dominant kernel (bin with the largest summed kernel time)
+    tot_ms = [sum(s["kernel_ms"][b] for s in stats) for b in range(4)]
+    dom = max(range(4), key=lambda b: tot_ms[b])
+    byts = sum(algorithmic_bytes(s, dom, weighted) for s in stats)
+    achieved = byts / (tot_ms[dom] / 1e3) / 1e9 if tot_ms[dom] > 0 else 0.0
+    peak, peak_src = peaks()
+    st0 = stats[-1]
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": None, "kernel": f"k_{BINS[dom]} (bin {BINS[dom]})",
+            "peak_source": peak_src,
+            "share_of_step": round(tot_ms[dom] / (ms * args.steps), 4),
+            "algorithmic_bytes_per_run": int(byts / args.steps),
+            "kernel_ms_per_run": round(tot_ms[dom] / args.steps, 3)}
+
+    line = {"metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": args.config, "N": N, "M": M, "weights": args.weights,
+                       "generator_seconds": round(t_gen, 1), "scale": args.scale,
+                       "l2": f"inputs ({(M * (8 if weighted else 4) + 8 * N) / 1e9:.1f} GB) larger than the 126 MB L2; no flush",
+                       "params": {"tolerance": 0.05, "max_iterations": 20, "pickless_period": 4, "mode": "async"},
+                       "parallelism": "single GPU"},
+            "iterations": st0["iterations"], "converged": st0["converged"], "changed": st0["changed"],
+            "modularity": q,
+            "bins": {BINS[b]: {"vertices": st0["bin_vertices"][b], "edges": st0["bin_edges"][b],
+                               "kernel_ms_per_run": round(tot_ms[b] / args.steps, 3)} for b in range(4)},
+            "roofline": roof, "gpu_launches": launches, "clocks": ck,
+            "context": "paper: 3.0e9 edges/s on it-2004 (2.19B edges) on one A100 (PAPER.md:501)"}
+
+    if args.extra:
+        if weighted:
+            g2 = nl.Graph(g.offsets, g.indices, None)
+            for _ in range(2):
+                g2.run()
+            torch.cuda.synchronize()
+            ev0.record(stream)
+            for _ in range(args.steps):
+                g2.run()
+            ev1.record(stream)
+            torch.cuda.synchronize()
+            line["unit_weight_fastpath"] = {"value": M / (ev0.elapsed_time(ev1) / args.steps / 1e3), "unit": "edges/s"}
+            g2.close()
+
+    if not args.no_e2e:
+        line["e2e"] = e2e(args, g, weights, gg)
+    if not args.no_cpu_baseline:
+        cb = cpu_baseline(args)
+        line["cpu_baseline"] = {k: cb[k] for k in ("value", "unit", "cores", "kind", "sample")}
+    print(json.dumps(line), flush=True)
+    gg.close()
+    return 0
+
+
+def e2e(args, g, weights, gg_dev):
+    """Same metric through the public C ABI with HOST buffers: each step
+    copies the CSR from pinned host memory (nulpa_create, memkind HOST), runs
+    nu-LPA (nulpa_run) and reads the labels back (nulpa_labels to host)."""
+    import torch
+    import paper_conf_ipps_sahunk25_b200 as nl
+    off_h = g.offsets.to("cpu").pin_memory()
+    idx_h = g.indices.to("cpu").pin_memory()
+    w_h = None if weights is None else weights.to("cpu").pin_memory()
+    lab_h = torch.empty(g.N, dtype=torch.int32).pin_memory()
+    h2d = off_h.numel() * 8 + idx_h.numel() * 4 + (0 if w_h is None else w_h.numel() * 4)
+    d2h = lab_h.numel() * 4
+    steps = max(1, min(args.steps, 3))
+    times = []
+    for it in range(steps + 1):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        h = nl.nulpa_create(off_h, idx_h, w_h)
+        nl.nulpa_run(h, nl.nulpa_default_params())
+        nl.nulpa_labels(h, lab_h)
+        torch.cuda.synchronize()
+        t1 = time.perf_counter()
+        nl.nulpa_destroy(h)
+        if it > 0:            # first one warms the allocator
+            times.append(t1 - t0)
+    sec = sum(times) / len(times)
+    return {"value": g.M / sec, "unit": "edges/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "ms_per_step": sec * 1e3, "steps": len(times)}
+
+
+def run_distributed(args, rank, world, local):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_sahunk25_b200 import distributed as D
+    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    g = make_graph(args, "cuda")
+    weights = torch.ones(g.M, dtype=torch.float32, device="cuda") if args.weights == "ones" else (
+        g.weights if args.weights == "random" else None)
+    shard = D.shard_graph(g.offsets, g.indices, weights, rank, world)
+    del g, weights
+    torch.cuda.empty_cache()
+    runner = D.CudaShardRunner(shard)
+    for _ in range(args.warmup):
+        D.lpa_distributed(runner)
+    torch.cuda.synchronize()
+    dist.barrier()
+    clocks = Clocks(local)
+    clocks.start()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    dist.barrier()
+    ev0.record()
+    res = None
+    for _ in range(args.steps):
+        res = D.lpa_distributed(runner)
+    ev1.record()
+    torch.cuda.synchronize()
+    dist.barrier()
+    ck = clocks.stop()
+    ms = torch.tensor([ev0.elapsed_time(ev1) / args.steps], dtype=torch.float64, device="cuda")
+    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms = float(ms.item())
+    q = D.modularity_distributed(runner)
+    if rank == 0:
+        line = {"metric": METRIC, "value": shard.M_global / (ms / 1e3), "unit": "edges/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": args.config, "N": shard.N_global, "M": shard.M_global, "weights": args.weights,
+                           "parallelism": f"vertex range split by edge count over {world} GPUs, NCCL all-gather of labels per sweep"},
+                "iterations": res["iterations"], "changed": res["changed"], "modularity": q,
+                "gpu_launches": res["launches"] * args.steps, "clocks": ck}
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,180 @@
+/*
+ * nulpa.h -- C ABI of the B200-native nu-LPA hot path.
+ *
+ * nu-LPA (PAPER.md, Sahu): asynchronous label propagation with a per-vertex
+ * open-addressing hashtable (float32 values, hybrid quadratic-double
+ * probing), the Pick-Less rule every rho iterations, vertex pruning, and a
+ * tolerance-based stop (Algorithm 1; Algorithm 2,
+ * PAPER.md:368-406), plus modularity (Eq. 1).
+ *
+ * Conventions for every entry point
+ *   - Return value: NULPA_OK (0) on success, a positive NULPA_E* code on
+ *     failure; nulpa_last_error() then describes the failure (thread-local
+ *     string owned by the library, valid until the next call on the thread).
+ *     No entry point aborts the process or falls back to the CPU.
+ *   - Graphs are CSR: offsets[n_rows+1] int64 (offsets[0]
+ *     must be 0), indices[M] int32 global vertex IDs in [0, n_global),
+ *     weights[M] float32 >= 0 or NULL for unit weights.
+ *     Undirected graphs store both directions.  Self-loops are skipped when
+ *     accumulating.
+ *   - `memkind` says where a pointer lives: NULPA_MEM_HOST (pageable or
+ *     pinned host memory) or NULPA_MEM_DEVICE (CUDA device memory on the
+ *     current device).
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  All device work of a handle is enqueued on the stream given
+ *     to nulpa_create; calls that return host results synchronise it.
+ *   - Labels are int32 community IDs; after nulpa_run they are vertex IDs.
+ */
+#ifndef NULPA_H
+#define NULPA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define NULPA_OK 0
+#define NULPA_EINVAL 1   /* bad argument (null pointer, size, range)        */
+#define NULPA_ECUDA 2    /* a CUDA runtime call or kernel launch failed      */
+#define NULPA_ENOMEM 3   /* device or pinned-host allocation failed          */
+#define NULPA_ESTATE 4   /* call not valid in the handle's current state     */
+
+#define NULPA_MEM_HOST 0
+#define NULPA_MEM_DEVICE 1
+
+#define NULPA_ASYNC 0    /* production mode: one label vector, in-place writes (PAPER.md:173 (1)) */
+#define NULPA_SYNC 1     /* deterministic Jacobi mode: reads previous sweep's labels (north star) */
+
+typedef struct nulpa_graph nulpa_graph;
+
+/* Parameters of nulpa_run / nulpa_sweep.  nulpa_default_params() fills the
+ * paper's values: tau = 0.05, 20 iterations, Pick-Less every 4 iterations
+ * (PAPER.md:173), asynchronous mode, B200 switch degrees. */
+typedef struct nulpa_params {
+    double tolerance;            /* tau: stop when not PL and dN/N < tau      */
+    int32_t max_iterations;      /* MAX_ITERATIONS                            */
+    int32_t pickless_period;     /* rho: PL when l mod rho == 0; <= 0 disables PL (R10)       */
+    int32_t mode;                /* NULPA_ASYNC or NULPA_SYNC                                 */
+    int32_t switch_degree;       /* degree >= this -> warp-per-vertex instead of thread-per-vertex
+                                    (the paper's SWITCH_DEGREE; B200 default 16) */
+    int32_t block_degree;        /* degree >= this -> block-per-vertex (shared-memory table)  */
+    int32_t giant_degree;        /* degree >= this -> multi-CTA, global-memory table          */
+    int32_t reset;               /* 1: C <- [0..N) and all vertices unprocessed first;
+                                    0: continue from the current labels / flags               */
+    int32_t timing;              /* 1: time every kernel with CUDA events (nulpa_get_stats)   */
+    int32_t tie_rule;            /* order among labels of equal weight (R6):
+                                    NULPA_TIE_SMALLEST (0): smallest label (north star);
+                                    NULPA_TIE_SLOT (1): first in the table's slot order -- smallest
+                                    home slot k mod p1, then smallest label (PAPER.md:173
+                                    "selects the first label with the highest associated weight") */
+    int32_t bin_order;           /* 1 (default): thread, warp, block, giant bins in that order
+                                    within a sweep (hubs last); 0: giant, block, warp, thread    */
+} nulpa_params;
+
+#define NULPA_TIE_SMALLEST 0
+#define NULPA_TIE_SLOT 1
+
+/* Statistics of the last nulpa_run (or accumulated nulpa_sweep calls since
+ * the last reset).  Bins: 0 thread, 1 warp, 2 block, 3 giant. */
+typedef struct nulpa_stats {
+    int32_t iterations;                /* iterations performed by the last nulpa_run   */
+    int32_t converged;                 /* 1 if stopped by the tolerance test           */
+    int64_t changed[64];               /* dN of iteration l (l < 64)                   */
+    int64_t vertices_processed[4];     /* per bin, summed over iterations              */
+    int64_t edges_scanned[4];          /* per bin, summed over iterations              */
+    int64_t vertices_changed[4];       /* per bin, summed over iterations              */
+    int64_t changed_edges[4];          /* per bin: CSR entries of changed vertices      */
+    double kernel_ms[4];               /* per bin, summed (timing=1 only)              */
+    int32_t launches[4];               /* kernel launches per bin                      */
+    int32_t other_launches;            /* init / copy / bookkeeping kernels            */
+    int64_t bin_vertices[4];           /* vertices in each degree bin                  */
+    int64_t bin_edges[4];              /* CSR entries of the vertices in each bin      */
+    double run_ms;                     /* wall time of nulpa_run on the stream (events) */
+} nulpa_stats;
+
+void nulpa_default_params(nulpa_params *p);
+
+/* Create a handle over a CSR graph or a row shard of one.
+ *   offsets  : n_rows+1 int64 prefix sums into indices/weights (offsets[0]==0)
+ *   indices  : offsets[n_rows] int32 neighbour IDs (global, < n_global)
+ *   weights  : offsets[n_rows] float32 (>= 0, R12) or NULL for unit weights
+ *   n_rows   : rows in this CSR (= vertices this handle sweeps)
+ *   n_global : vertices of the whole graph (length of the label array);
+ *              single-GPU: n_global == n_rows
+ *   row_begin: global ID of row 0 (shards: rows are vertices
+ *              [row_begin, row_begin+n_rows)); single-GPU: 0
+ *   memkind  : where offsets/indices/weights live.  DEVICE arrays are
+ *              BORROWED (the caller keeps them alive and unchanged until
+ *              nulpa_destroy); HOST arrays are copied to device memory owned
+ *              by the handle (copy enqueued on `stream`; the host arrays may
+ *              be reused once nulpa_create returns).
+ *   stream   : cudaStream_t for all work of this handle.
+ * Builds the degree-binned frontier (row a1) with the default switch degrees;
+ * nulpa_run rebuilds it if other switch degrees are requested.
+ * Labels start as C = [0..n_global), all vertices unprocessed. */
+int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *weights,
+                 int64_t n_rows, int64_t n_global, int64_t row_begin, int memkind,
+                 void *stream, nulpa_graph **out);
+
+/* Use caller-owned device buffers for the label vector (n_global int32) and
+ * the "unprocessed" flags (n_global uint8, nonzero = unprocessed) instead of
+ * the handle's own (multi-GPU driver: the replicated label array is a torch
+ * tensor exchanged by NCCL).  Their contents are adopted as the current
+ * state.  Borrowed until nulpa_destroy. */
+int nulpa_bind_state(nulpa_graph *g, int32_t *labels_device, uint8_t *flags_device);
+
+/* Run Algorithm 1's lpa() loop with `params` (NULL =
+ * defaults) and fill *stats (may be NULL).  Synchronises the stream once per
+ * iteration (the tolerance test needs dN on the host). */
+int nulpa_run(nulpa_graph *g, const nulpa_params *params, nulpa_stats *stats);
+
+/* One lpaMove over this handle's rows with Pick-Less on
+ * or off; *changed receives dN (may be NULL: then the call does not
+ * synchronise).  params supplies mode and switch degrees (NULL = defaults). */
+int nulpa_sweep(nulpa_graph *g, int pickless, const nulpa_params *params, int64_t *changed);
+
+/* Reset to C = [0..n_global), all unprocessed. */
+int nulpa_reset(nulpa_graph *g);
+
+/* Copy the current labels (n_global int32) to `out` in `memkind` memory. */
+int nulpa_labels(nulpa_graph *g, int32_t *out, int memkind);
+
+/* Overwrite the labels (n_global int32 from `in` in `memkind` memory) and
+ * the unprocessed flags (n_global uint8, or NULL = all unprocessed). */
+int nulpa_set_labels(nulpa_graph *g, const int32_t *in, const uint8_t *flags, int memkind);
+
+/* Copy the unprocessed flags (n_global uint8) to `out`. */
+int nulpa_flags(nulpa_graph *g, uint8_t *out, int memkind);
+
+/* Modularity Q of `labels` (n_global int32 in [0, n_global), memkind; NULL =
+ * the handle's current labels), Eq. 1 second form (R11), float64
+ * accumulation.  Requires a whole graph (n_rows == n_global). */
+int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double *q);
+
+/* Shard pieces of the modularity for the multi-GPU driver: adds this
+ * shard's intra-community weight to *sigma_intra, its total weight to
+ * *two_m, and K_i into Sigma_device[labels[i]] (n_global float64, device). */
+int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, double *sigma_intra,
+                             double *two_m, double *Sigma_device);
+/* Q = sigma_intra/two_m - sum_c (Sigma_c/two_m)^2 over a device Sigma. */
+int nulpa_modularity_finish(nulpa_graph *g, const double *Sigma_device, double sigma_intra,
+                            double two_m, double *q);
+
+int nulpa_get_stats(nulpa_graph *g, nulpa_stats *out);
+
+/* Device pointers of the current label / flag vectors (for zero-copy
+ * wrapping by the binding).  Valid until the next nulpa_* call. */
+int nulpa_state_pointers(nulpa_graph *g, int32_t **labels_device, uint8_t **flags_device);
+
+int nulpa_destroy(nulpa_graph *g);
+
+const char *nulpa_last_error(void);
+
+/* Library version string ("nulpa <semver> sm_100a"). */
+const char *nulpa_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NULPA_H */

@@ -1,0 +1,1985 @@
+// nulpa.cu -- B200 (sm_100a) implementation of the nu-LPA hot path behind the
+// C ABI declared in include/nulpa.h.
+//
+// Paper: PAPER.md (Sahu, nu-LPA).  Algorithm 1 is the
+// sweep/loop structure, Algorithm 2 the per-vertex
+// hashtable, Eq. 1 the modularity.  Readings R1..R12 are
+// listed in DESIGN.md.  This file shares no code with oracle/.
+//
+// Layout in HBM:
+//   offsets  int64 [n_rows+1]   indices int32 [M]   weights float32 [M] | null
+//   labels   int32 [n_global]   flags   uint8 [n_global] (1 = unprocessed)
+//   bin lists int32 (row ids), one per degree bin, stable in row order
+//   giant tables: int32 keys / float32 values / int32 occupied-slot lists,
+//   one region of p1 = nextPow2(D)-1 slots per giant vertex.
+//
+// Kernels of one sweep (lpaMove), launched on the handle's stream in order
+// giant -> block -> warp -> thread (largest work first):
+//   k_giant_snapshot / k_giant_accumulate / k_giant_finalize / k_giant_mark
+//   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
+//   k_warp    one warp per vertex, shared-memory table (<= 255 slots)
+//   k_thread  one thread per vertex, labels in registers (degree < 32)
+
+#include "nulpa.h"
+
+#include <cuda_runtime.h>
+#include <cub/device/device_scan.cuh>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+namespace {
+
+constexpr int32_t kEmpty = -1;           // phi
+constexpr int kMaxRetries = 16;          // R5
+constexpr int kMaxIter = 64;             // counters kept per iteration
+constexpr int kCtr = 24;                 // counters per iteration
+// counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
+
+constexpr int kWarpThreads = 256;        // k_warp: 8 warps per CTA
+constexpr int kWarpCap = 256;            // slots per warp table (degree <= 255 -> p1 <= 255)
+constexpr int kBlockThreads = 512;       // k_block / giant kernels
+constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
+constexpr int kGiantChunk = 4096;        // edges per giant chunk
+constexpr int kGiantCap = 8192;          // slots of a chunk table (4096 edges -> p1 = 8191)
+constexpr int kThreadThreads = 256;
+
+thread_local std::string g_err;
+
+int fail(int code, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CU(call)                                                                             \
+    do {                                                                                     \
+        cudaError_t e_ = (call);                                                             \
+        if (e_ != cudaSuccess)                                                               \
+            return fail(e_ == cudaErrorMemoryAllocation ? NULPA_ENOMEM : NULPA_ECUDA,        \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,    \
+                        __LINE__);                                                           \
+    } while (0)
+
+#define CHECK(x)                              \
+    do {                                      \
+        int r_ = (x);                         \
+        if (r_ != NULPA_OK) return r_;        \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// device helpers
+// ---------------------------------------------------------------------------
+
+// Lemire's fastmod for 32-bit operands: a mod d with M = floor((2^64-1)/d)+1.
+__device__ __forceinline__ uint32_t fastmod(uint32_t a, uint64_t M, uint32_t d) {
+    uint64_t low = M * a;
+    return (uint32_t)__umul64hi(low, d);
+}
+
+// R1: capacity p1 = nextPow2(D) - 1 with nextPow2 strictly greater than D;
+// R3: p2 = 2*p1 + 1.
+__host__ __device__ __forceinline__ uint32_t capacity_p1(uint32_t D) {
+#ifdef __CUDA_ARCH__
+    return D == 0 ? 0u : (uint32_t)((2ull << (31 - __clz(D))) - 1);
+#else
+    uint64_t p = 1;
+    while (p <= D) p <<= 1;
+    return (uint32_t)(p - 1);
+#endif
+}
+
+// Capacities are Mersenne numbers p = 2^a - 1 (R1, R3), so the fastmod
+// magic of every p1 / p2 comes from a compile-time table indexed by a.
+struct MagicTable {
+    uint64_t m[34];
+    constexpr MagicTable() : m() {
+        m[0] = 0;
+        for (int a = 1; a < 34; ++a) m[a] = UINT64_C(0xFFFFFFFFFFFFFFFF) / ((UINT64_C(1) << a) - 1) + 1;
+    }
+};
+__constant__ MagicTable c_magic = MagicTable();
+
+struct Hash {
+    uint32_t p1, p2;
+    uint64_t m1, m2;
+    __device__ __forceinline__ void init(uint32_t degree) {
+        const int a = degree ? 32 - __clz(degree) : 0;   // nextPow2(D) = 2^a (R1)
+        p1 = a ? (uint32_t)((UINT64_C(1) << a) - 1) : 0u;
+        p2 = 2 * p1 + 1;                                  // R3
+        m1 = c_magic.m[a];
+        m2 = c_magic.m[a + 1];
+    }
+};
+
+// Tie order among labels of equal weight (R6).  Rule 0 (north star):
+// smallest label.  Rule 1 ("the first label with the highest
+// associated weight", read as first in the table's slot order): smallest home
+// slot k mod p1, then smallest label.  Both are independent of insertion
+// order.  rank(k) maps k to a 32-bit integer whose order is the tie order:
+// rule 1 uses (k mod p1) * Q + (k div p1) with Q = floor((2^31-1)/p1) + 1,
+// a bijection onto [0, p1*Q) < 2^32; (k div p1) is the exact division
+// (k - k mod p1) * p1^-1 mod 2^32 (p1 = 2^a - 1 is odd).
+struct TieOrder {
+    int rule;
+    uint32_t p1, Q, inv;
+    uint64_t m1;
+    __device__ __forceinline__ void init(int r, const Hash &h) {
+        rule = r;
+        p1 = h.p1;
+        m1 = h.m1;
+        if (r) {
+            Q = p1 ? 0x7FFFFFFFu / p1 + 1 : 1;
+            uint32_t x = p1;                       // Newton: x <- x (2 - p1 x)
+#pragma unroll
+            for (int i = 0; i < 5; ++i) x *= 2u - p1 * x;
+            inv = x;
+        }
+    }
+    __device__ __forceinline__ uint32_t rank(int32_t k) const {
+        if (!rule) return (uint32_t)k;
+        uint32_t home = fastmod((uint32_t)k, m1, p1);
+        return home * Q + ((uint32_t)k - home) * inv;
+    }
+    __device__ __forceinline__ int32_t unrank(uint32_t t) const {
+        if (!rule) return (int32_t)t;
+        uint32_t home = t / Q;
+        return (int32_t)((t - home * Q) * p1 + home);
+    }
+};
+
+// hashtableAccumulate, Algorithm 2, the SHARED branch:
+// atomicCAS claims an empty slot, atomicAdd accumulates.  Works on shared or
+// global memory (generic addressing).  i and delta_i are kept reduced mod p1
+// (same slots); R5 linear continuation after kMaxRetries probes.
+// Returns true if the key newly claimed a slot (*slot_out = slot).
+__device__ __forceinline__ bool ht_accumulate(int32_t *Hk, float *Hv, const Hash &h, int32_t k,
+                                              float v, uint32_t *slot_out = nullptr) {
+    const uint32_t p1 = h.p1;
+    uint32_t i = fastmod((uint32_t)k, h.m1, p1);
+    uint32_t di = p1 > 1 ? 1u : 0u;
+    uint32_t km = fastmod((uint32_t)k, h.m2, h.p2);
+    if (km >= p1) km -= p1;
+    if (km >= p1) km -= p1;
+    for (int t = 0; t < kMaxRetries; ++t) {
+        int32_t cur = *((volatile int32_t *)&Hk[i]);
+        if (cur == k || cur == kEmpty) {
+            int32_t old = cur == k ? k : atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty || old == k) {
+                atomicAdd(&Hv[i], v);
+                if (slot_out) *slot_out = i;
+                return old == kEmpty;
+            }
+        }
+        i += di;
+        if (i >= p1) i -= p1;
+        di = 2 * di + km;            // < 2p1 + p1
+        if (di >= p1) di -= p1;
+        if (di >= p1) di -= p1;
+    }
+    for (uint32_t t = 0; t < p1; ++t) {     // R5
+        int32_t cur = *((volatile int32_t *)&Hk[i]);
+        if (cur == k || cur == kEmpty) {
+            int32_t old = cur == k ? k : atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty || old == k) {
+                atomicAdd(&Hv[i], v);
+                if (slot_out) *slot_out = i;
+                return old == kEmpty;
+            }
+        }
+        i = i + 1 == p1 ? 0 : i + 1;
+    }
+    return false;  // unreachable: distinct keys <= D <= p1
+}
+
+// Algorithm 2's probe sequence without the value update: find the slot
+// holding k or claim an empty one with atomicCAS (R5 linear continuation).
+__device__ __forceinline__ uint32_t ht_claim(int32_t *Hk, const Hash &h, int32_t k) {
+    const uint32_t p1 = h.p1;
+    uint32_t i = fastmod((uint32_t)k, h.m1, p1);
+    uint32_t di = p1 > 1 ? 1u : 0u;
+    uint32_t km = fastmod((uint32_t)k, h.m2, h.p2);
+    if (km >= p1) km -= p1;
+    if (km >= p1) km -= p1;
+    for (int t = 0; t < kMaxRetries; ++t) {
+        int32_t cur = *((volatile int32_t *)&Hk[i]);
+        if (cur == k) return i;
+        if (cur == kEmpty) {
+            int32_t old = atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty || old == k) return i;
+        }
+        i += di;
+        if (i >= p1) i -= p1;
+        di = 2 * di + km;
+        if (di >= p1) di -= p1;
+        if (di >= p1) di -= p1;
+    }
+    for (uint32_t t = 0; t < p1; ++t) {
+        int32_t cur = *((volatile int32_t *)&Hk[i]);
+        if (cur == k) return i;
+        if (cur == kEmpty) {
+            int32_t old = atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty || old == k) return i;
+        }
+        i = i + 1 == p1 ? 0 : i + 1;
+    }
+    return 0;  // unreachable: distinct keys <= D <= p1
+}
+
+// Sum of `x` over the lanes of this lane's match_any group `grp`, delivered
+// to the group's lowest lane (rank 0): a pairwise tree over the members in
+// lane (= CSR) order.  The member d ranks ahead is found by pointer jumping
+// (nxt <- nxt[nxt] doubles the distance each step), two shuffles per level.
+// maxn (warp-uniform) = largest group size.
+__device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn) {
+    const int lane = threadIdx.x & 31;
+    const unsigned rank = __popc(grp & ((1u << lane) - 1));
+    const unsigned above = lane == 31 ? 0u : grp & (0xFFFFFFFEu << lane);
+    int nxt = above ? __ffs(above) - 1 : 32;               // member 1 ahead (32 = none)
+    for (unsigned d = 1; d < maxn; d <<= 1) {
+        const float y = __shfl_sync(0xFFFFFFFFu, x, nxt & 31);
+        const int n2 = __shfl_sync(0xFFFFFFFFu, nxt, nxt & 31);
+        if ((rank & (2 * d - 1)) == 0 && nxt < 32) x = __fadd_rn(x, y);
+        nxt = nxt < 32 ? n2 : 32;                          // member 2d ahead
+    }
+    return x;
+}
+
+// One 32-edge batch of a warp against the warp's PRIVATE table: lanes
+// holding the same label (match_any) are folded onto their lowest lane (the
+// leader), which claims the label's slot (Algorithm 2 probing, atomicCAS on
+// the key) and adds the group's weight with a plain shared-memory
+// read-modify-write -- no other lane of the batch touches that slot, and
+// batches are ordered by __syncwarp, so no float atomics are needed (the GPU
+// has no native shared-memory float atomicAdd).  Unit weights: the group
+// weight is the member count, exact.  key == kEmpty marks an idle lane.
+template <bool W>
+__device__ __forceinline__ void warp_batch_accumulate(int32_t *Hk, float *Hv, const Hash &h, int32_t key, float w) {
+    const int lane = threadIdx.x & 31;
+    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+    const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
+    float sum;
+    if (W) {
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
+    } else {
+        sum = (float)__popc(grp);
+    }
+    if (leader) {
+        const uint32_t slot = ht_claim(Hk, h, key);
+        Hv[slot] = __fadd_rn(Hv[slot], sum);
+    }
+    __syncwarp();
+}
+
+// The same folding for a table shared by several warps (block / giant
+// kernels): the leader adds its group's sum with one shared-memory
+// atomicAdd (a CAS loop on this GPU, now contended by at most one lane per
+// warp and label).
+template <bool W>
+__device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float *Hv, const Hash &h, int32_t key,
+                                                             float w) {
+    const int lane = threadIdx.x & 31;
+    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+    const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
+    float sum;
+    if (W) {
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
+    } else {
+        sum = (float)__popc(grp);
+    }
+    if (leader) atomicAdd(&Hv[ht_claim(Hk, h, key)], sum);
+}
+
+// (weight, tie rank) packed so that an unsigned max gives the largest weight
+// and, among equal weights, the label first in tie order (R6; R12: weights
+// >= 0 so IEEE bit patterns order like the values).  0 = no candidate.
+__device__ __forceinline__ uint64_t pack_cand(float w, int32_t k, const TieOrder &to) {
+    return ((uint64_t)__float_as_uint(w) << 32) | (uint64_t)(0xFFFFFFFFu - to.rank(k));
+}
+__device__ __forceinline__ int32_t cand_label(uint64_t c, const TieOrder &to) {
+    return to.unrank(0xFFFFFFFFu - (uint32_t)(c & 0xFFFFFFFFu));
+}
+__device__ __forceinline__ uint64_t warp_max_u64(uint64_t x) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        uint64_t y = __shfl_xor_sync(0xFFFFFFFFu, x, o);
+        x = y > x ? y : x;
+    }
+    return x;
+}
+
+// The move rule, PAPER.md:344 (R7: no candidate -> keep the label).
+__device__ __forceinline__ bool accept_move(int32_t cstar, int32_t ci, int pickless) {
+    return cstar != kEmpty && cstar != ci && (!pickless || cstar <= ci);
+}
+
+struct SweepArgs {
+    const int64_t *__restrict__ offsets;
+    const int32_t *__restrict__ indices;
+    const float *__restrict__ weights;
+    const int32_t *lab_in;     // async: == lab_out
+    int32_t *lab_out;
+    uint8_t *flag_in;          // async: == flag_out
+    uint8_t *flag_out;
+    int64_t row_begin;
+    int pickless;
+    int tie_rule;
+    unsigned long long *ctr;   // kCtr counters of this iteration
+};
+
+// Warp-aggregated (ballot / redux) then CTA-aggregated changed-vertex,
+// processed-vertex and edge counters: one set of global atomics per CTA.
+// bctr: 4 shared counters zeroed before the first __syncthreads.
+__device__ __forceinline__ void block_count(unsigned long long *ctr, unsigned long long *bctr, int bin, bool act,
+                                            bool changed, uint32_t edges) {
+    unsigned m_act = __ballot_sync(0xFFFFFFFFu, act);
+    unsigned m_ch = __ballot_sync(0xFFFFFFFFu, changed);
+    uint32_t e = __reduce_add_sync(0xFFFFFFFFu, edges);
+    uint32_t ec = __reduce_add_sync(0xFFFFFFFFu, changed ? edges : 0u);
+    if ((threadIdx.x & 31) == 0 && m_act) {
+        atomicAdd(&bctr[0], (unsigned long long)__popc(m_act));
+        atomicAdd(&bctr[1], (unsigned long long)e);
+        atomicAdd(&bctr[2], (unsigned long long)__popc(m_ch));
+        atomicAdd(&bctr[3], (unsigned long long)ec);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && bctr[0]) {
+        atomicAdd(&ctr[1 + bin], bctr[0]);
+        atomicAdd(&ctr[5 + bin], bctr[1]);
+        if (bctr[2]) {
+            atomicAdd(&ctr[0], bctr[2]);
+            atomicAdd(&ctr[9 + bin], bctr[2]);
+            atomicAdd(&ctr[13 + bin], bctr[3]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// thread-per-vertex kernel (degree < switch_degree <= 33), PAPER.md:241-243:
+// "only a single thread operates on the hashtable.  This eliminates the need
+// for atomic operations".  With at most MAXD neighbours the table lives in
+// registers: the weight of label lab[k] is the sum over m of w[m] where
+// lab[m] == lab[k], taken in CSR order (bit-identical to a sequential
+// float32 hashtable accumulation).
+// ---------------------------------------------------------------------------
+template <bool SYNC, bool W, int MAXD>
+__global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const int32_t *__restrict__ list,
+                                                           int64_t n) {
+    __shared__ unsigned long long bctr[4];
+    if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
+    __syncthreads();
+    int64_t t = (int64_t)blockIdx.x * kThreadThreads + threadIdx.x;
+    bool act = false, changed = false;
+    uint32_t deg = 0;
+    if (t < n) {
+        int32_t r = list[t];
+        int64_t v = r + a.row_begin;
+        if (a.flag_in[v]) {
+            act = true;
+            if (!SYNC) a.flag_in[v] = 0;                 // mark i as processed
+            int64_t o = a.offsets[r];
+            deg = (uint32_t)(a.offsets[r + 1] - o);
+            int32_t lab[MAXD];
+            float w[MAXD];
+#pragma unroll
+            for (int k = 0; k < MAXD; ++k) {
+                lab[k] = kEmpty;
+                w[k] = 0.0f;
+                if (k < (int)deg) {
+                    int32_t j = a.indices[o + k];
+                    if (j != (int32_t)v) {                // "if j = i continue"
+                        lab[k] = a.lab_in[j];
+                        w[k] = W ? a.weights[o + k] : 1.0f;
+                    }
+                }
+            }
+            Hash h;
+            h.init(deg);
+            TieOrder to;
+            to.init(a.tie_rule, h);
+            uint64_t best = 0;
+#pragma unroll
+            for (int k = 0; k < MAXD; ++k) {
+                if (k >= (int)deg) break;
+                if (lab[k] == kEmpty) continue;
+                float s = 0.0f;
+#pragma unroll
+                for (int m = 0; m < MAXD; ++m) {
+                    if (m >= (int)deg) break;
+                    s = __fadd_rn(s, lab[m] == lab[k] ? w[m] : 0.0f);
+                }
+                uint64_t c = pack_cand(s, lab[k], to);
+                best = c > best ? c : best;
+            }
+            int32_t ci = a.lab_in[v];
+            int32_t cs = best ? cand_label(best, to) : kEmpty;
+            if (accept_move(cs, ci, a.pickless)) {
+                a.lab_out[v] = cs;
+                changed = true;
+                for (uint32_t k = 0; k < deg; ++k) a.flag_out[a.indices[o + k]] = 1;
+            }
+        }
+    }
+    block_count(a.ctr, bctr, 0, act, changed, act ? deg : 0);
+}
+
+// ---------------------------------------------------------------------------
+// warp-per-vertex kernel: one 32-lane warp per vertex, the vertex's table
+// (p1 <= 255 slots) in shared memory, persistent grid-stride over the bin.
+// ---------------------------------------------------------------------------
+template <bool SYNC, bool W>
+__global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_t *__restrict__ list,
+                                                       int64_t n) {
+    __shared__ int32_t sk[kWarpThreads / 32][kWarpCap];
+    __shared__ float sv[kWarpThreads / 32][kWarpCap];
+    __shared__ unsigned long long bctr[4];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int32_t *Hk = sk[wid];
+    float *Hv = sv[wid];
+    for (int s = lane; s < kWarpCap; s += 32) {
+        Hk[s] = kEmpty;
+        Hv[s] = 0.0f;
+    }
+    if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
+    __syncthreads();
+    unsigned long long c_act = 0, c_edges = 0, c_ch = 0, c_che = 0;   // lane 0's tallies
+    const int64_t nw = (int64_t)gridDim.x * (kWarpThreads / 32);
+    const int64_t nchunks = (n + 31) / 32;
+    // Each warp takes chunks of 32 consecutive bin entries: the metadata of
+    // all 32 vertices (row, flag, offsets, own label) is fetched in one
+    // round trip, lane k holding vertex k; the warp then walks the active ones.
+    for (int64_t c = (int64_t)blockIdx.x * (kWarpThreads / 32) + wid; c < nchunks; c += nw) {
+        const int64_t t = c * 32 + lane;
+        int32_t r = 0, ci = 0;
+        int f = 0;
+        int64_t o = 0;
+        uint32_t deg = 0;
+        if (t < n) {
+            r = list[t];
+            f = a.flag_in[r + a.row_begin];
+        }
+        if (f) {
+            o = a.offsets[r];
+            deg = (uint32_t)(a.offsets[r + 1] - o);
+            ci = a.lab_in[r + a.row_begin];
+            if (!SYNC) a.flag_in[r + a.row_begin] = 0;     // mark i as processed
+        }
+        unsigned act = __ballot_sync(0xFFFFFFFFu, f != 0);
+        while (act) {
+            const int k = __ffs(act) - 1;
+            act &= act - 1;
+            const int32_t rk = __shfl_sync(0xFFFFFFFFu, r, k);
+            const int64_t ok = __shfl_sync(0xFFFFFFFFu, o, k);
+            const uint32_t dk = __shfl_sync(0xFFFFFFFFu, deg, k);
+            const int32_t cik = __shfl_sync(0xFFFFFFFFu, ci, k);
+            const int64_t vk = rk + a.row_begin;
+            Hash h;
+            h.init(dk);
+            // the first 64 entries of the row stay in registers (degree < 64
+            // covers most vertices); indices/weights first, then all the
+            // neighbour labels: two dependent round trips per vertex
+            const bool v0 = (uint32_t)lane < dk, v1 = (uint32_t)(lane + 32) < dk;
+            const int32_t j0 = v0 ? a.indices[ok + lane] : -1;
+            const int32_t j1 = v1 ? a.indices[ok + 32 + lane] : -1;
+            float w0 = 0.0f, w1 = 0.0f;
+            if (W) {
+                if (v0) w0 = a.weights[ok + lane];
+                if (v1) w1 = a.weights[ok + 32 + lane];
+            }
+            const int32_t k0 = (j0 >= 0 && j0 != (int32_t)vk) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
+            const int32_t k1 = (j1 >= 0 && j1 != (int32_t)vk) ? a.lab_in[j1] : kEmpty;
+            warp_batch_accumulate<W>(Hk, Hv, h, k0, w0);
+            if (dk > 32) warp_batch_accumulate<W>(Hk, Hv, h, k1, w1);
+            for (uint32_t b = 64; b < dk; b += 64) {
+                const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
+                const int32_t i0 = u0 ? a.indices[ok + b + lane] : -1;
+                const int32_t i1 = u1 ? a.indices[ok + b + 32 + lane] : -1;
+                float x0 = 0.0f, x1 = 0.0f;
+                if (W) {
+                    if (u0) x0 = a.weights[ok + b + lane];
+                    if (u1) x1 = a.weights[ok + b + 32 + lane];
+                }
+                const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
+                const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
+                warp_batch_accumulate<W>(Hk, Hv, h, q0, x0);
+                if (b + 32 < dk) warp_batch_accumulate<W>(Hk, Hv, h, q1, x1);
+            }
+            TieOrder to;
+            to.init(a.tie_rule, h);
+            uint64_t best = 0;
+            for (uint32_t s = lane; s < h.p1; s += 32) {    // hashtableMaxKey + clear
+                const int32_t key = Hk[s];
+                if (key != kEmpty) {
+                    const uint64_t cd = pack_cand(Hv[s], key, to);
+                    best = cd > best ? cd : best;
+                    Hk[s] = kEmpty;
+                    Hv[s] = 0.0f;
+                }
+            }
+            best = warp_max_u64(best);
+            const int32_t cs = best ? cand_label(best, to) : kEmpty;
+            const bool changed = accept_move(cs, cik, a.pickless);
+            if (changed) {
+                if (lane == 0) a.lab_out[vk] = cs;
+                if (j0 >= 0) a.flag_out[j0] = 1;            // mark neighbours unprocessed
+                if (j1 >= 0) a.flag_out[j1] = 1;
+                for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[a.indices[ok + b]] = 1;
+            }
+            __syncwarp();
+            c_act += 1;
+            c_edges += dk;
+            c_ch += changed;
+            c_che += changed ? dk : 0;
+        }
+    }
+    if (lane == 0 && c_act) {
+        atomicAdd(&bctr[0], c_act);
+        atomicAdd(&bctr[1], c_edges);
+        atomicAdd(&bctr[2], c_ch);
+        atomicAdd(&bctr[3], c_che);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && bctr[0]) {
+        atomicAdd(&a.ctr[1 + 1], bctr[0]);
+        atomicAdd(&a.ctr[5 + 1], bctr[1]);
+        if (bctr[2]) {
+            atomicAdd(&a.ctr[0], bctr[2]);
+            atomicAdd(&a.ctr[9 + 1], bctr[2]);
+            atomicAdd(&a.ctr[13 + 1], bctr[3]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// tile kernel (the warp bin, switch_degree <= degree < block_degree): the
+// bin is cut into tiles of consecutive bin entries holding ~kTileE first
+// edges (<= kTileV vertices).  A CTA (8 warps) processes a tile in phases:
+//   1. metadata of all tile vertices (row, flag, offsets, own label) in one
+//      round trip, one thread per vertex; an exclusive scan places the
+//      active rows back to back in shared memory;
+//   2. the active rows' indices / weights are staged into shared memory with
+//      cp.async (LDGSTS, no register round trip; many copies in flight);
+//   3. the neighbour labels are gathered, ~9 independent loads per thread;
+//   4. each warp runs Algorithm 1's per-vertex body for its vertices from
+//      shared memory: fold the row into the warp-private table
+//      (warp_batch_accumulate), hashtableMaxKey, move rule, mark neighbours.
+// Global-memory latency is paid a few times per tile instead of per vertex.
+// ---------------------------------------------------------------------------
+constexpr int kTileThreads = 256;
+constexpr int kTileE = 2048;                 // first-edge budget of a tile
+constexpr int kTileV = 256;                  // vertices per tile (one per thread)
+constexpr int kTileSlots = kTileE + kWarpCap; // + the last vertex's degree (< 256)
+
+template <bool W>
+struct TileSmem {
+    int32_t hk[kTileThreads / 32][kWarpCap];
+    float hv[kTileThreads / 32][kWarpCap];
+    int32_t idx[kTileSlots];
+    int32_t lab[kTileSlots];
+    float w[W ? kTileSlots : 1];
+    int64_t o[kTileV];
+    int32_t r[kTileV];
+    int32_t deg[kTileV];
+    int32_t ci[kTileV];
+    int32_t pfx[kTileV + 1];
+    int32_t act[kTileV];
+    int32_t wsum[kTileThreads / 32];
+    int32_t nact;
+    unsigned long long bctr[4];
+};
+
+__device__ __forceinline__ void cp_async4(void *smem, const void *gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+template <bool SYNC, bool W>
+__global__ void __launch_bounds__(kTileThreads, 4) k_tile(SweepArgs a, const int32_t *__restrict__ list,
+                                                           const int32_t *__restrict__ tile_start, int64_t ntiles) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmem<W> &S = *reinterpret_cast<TileSmem<W> *>(smem_raw);
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    int32_t *Hk = S.hk[wid];
+    float *Hv = S.hv[wid];
+    for (int q = lane; q < kWarpCap; q += 32) {
+        Hk[q] = kEmpty;
+        Hv[q] = 0.0f;
+    }
+    if (tid < 4) S.bctr[tid] = 0;
+    unsigned long long c_act = 0, c_edges = 0, c_ch = 0, c_che = 0;   // lane 0's tallies
+    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int32_t k0 = tile_start[tile];
+        const int nv = tile_start[tile + 1] - k0;
+        // -- phase 1: metadata, one thread per vertex ------------------------
+        int32_t d = 0;
+        if (tid < nv) {
+            const int32_t r = list[k0 + tid];
+            const int64_t v = r + a.row_begin;
+            S.r[tid] = r;
+            if (a.flag_in[v]) {
+                const int64_t o = a.offsets[r];
+                d = (int32_t)(a.offsets[r + 1] - o);
+                S.o[tid] = o;
+                S.ci[tid] = a.lab_in[v];
+                if (!SYNC) a.flag_in[v] = 0;                // mark i as processed
+            }
+            S.deg[tid] = d;
+        }
+        // exclusive scan of active degrees + compaction of active slots
+        int32_t x = d;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const int32_t y = __shfl_up_sync(0xFFFFFFFFu, x, off);
+            if (lane >= off) x += y;
+        }
+        const unsigned am = __ballot_sync(0xFFFFFFFFu, d > 0);
+        if (lane == 31) S.wsum[wid] = x;
+        __shared__ int32_t wact[kTileThreads / 32];
+        if (lane == 0) wact[wid] = __popc(am);
+        __syncthreads();
+        int32_t base = 0, abase = 0;
+        for (int q = 0; q < wid; ++q) {
+            base += S.wsum[q];
+            abase += wact[q];
+        }
+        S.pfx[tid] = base + x - d;
+        if (d > 0) S.act[abase + __popc(am & ((1u << lane) - 1))] = tid;
+        if (tid == kTileThreads - 1) {
+            S.pfx[kTileV] = base + x;
+            S.nact = abase + __popc(am);
+        }
+        __syncthreads();
+        const int nact = S.nact;
+        const int32_t total = S.pfx[kTileV];
+        // -- phase 2: stage the active rows with cp.async --------------------
+        for (int q = wid; q < nact; q += kTileThreads / 32) {
+            const int kk = S.act[q];
+            const int64_t o = S.o[kk];
+            const int32_t dk = S.deg[kk], p0 = S.pfx[kk];
+            for (int e = lane; e < dk; e += 32) {
+                cp_async4(&S.idx[p0 + e], a.indices + o + e);
+                if (W) cp_async4(&S.w[p0 + e], a.weights + o + e);
+            }
+        }
+        cp_async_wait_all();
+        __syncthreads();
+        // -- phase 3: gather neighbour labels --------------------------------
+        for (int p = tid; p < total; p += 4 * kTileThreads) {
+            int32_t j[4], l[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) j[u] = p + u * kTileThreads < total ? S.idx[p + u * kTileThreads] : -1;
+#pragma unroll
+            for (int u = 0; u < 4; ++u) l[u] = j[u] >= 0 ? a.lab_in[j[u]] : kEmpty;
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (j[u] >= 0) S.lab[p + u * kTileThreads] = l[u];
+        }
+        __syncthreads();
+        // -- phase 4: per-vertex body, one warp per vertex -------------------
+        for (int q = wid; q < nact; q += kTileThreads / 32) {
+            const int kk = S.act[q];
+            const int64_t vk = S.r[kk] + a.row_begin;
+            const uint32_t dk = (uint32_t)S.deg[kk];
+            const int32_t p0 = S.pfx[kk];
+            Hash h;
+            h.init(dk);
+            for (uint32_t b = 0; b < dk; b += 32) {
+                int32_t key = kEmpty;
+                float w = 0.0f;
+                if (b + lane < dk) {
+                    const int32_t p = p0 + (int32_t)(b + lane);
+                    if (S.idx[p] != (int32_t)vk) {           // "if j = i continue"
+                        key = S.lab[p];
+                        if (W) w = S.w[p];
+                    }
+                }
+                warp_batch_accumulate<W>(Hk, Hv, h, key, w);
+            }
+            TieOrder to;
+            to.init(a.tie_rule, h);
+            uint64_t best = 0;
+            for (uint32_t sl = lane; sl < h.p1; sl += 32) { // hashtableMaxKey + clear
+                const int32_t key = Hk[sl];
+                if (key != kEmpty) {
+                    const uint64_t cd = pack_cand(Hv[sl], key, to);
+                    best = cd > best ? cd : best;
+                    Hk[sl] = kEmpty;
+                    Hv[sl] = 0.0f;
+                }
+            }
+            best = warp_max_u64(best);
+            const int32_t cs = best ? cand_label(best, to) : kEmpty;
+            const bool changed = accept_move(cs, S.ci[kk], a.pickless);
+            if (changed) {
+                if (lane == 0) a.lab_out[vk] = cs;
+                for (uint32_t b = lane; b < dk; b += 32) a.flag_out[S.idx[p0 + b]] = 1;   // mark neighbours
+            }
+            __syncwarp();
+            c_act += 1;
+            c_edges += dk;
+            c_ch += changed;
+            c_che += changed ? dk : 0;
+        }
+        __syncthreads();
+    }
+    if (lane == 0 && c_act) {
+        atomicAdd(&S.bctr[0], c_act);
+        atomicAdd(&S.bctr[1], c_edges);
+        atomicAdd(&S.bctr[2], c_ch);
+        atomicAdd(&S.bctr[3], c_che);
+    }
+    __syncthreads();
+    if (tid == 0 && S.bctr[0]) {
+        atomicAdd(&a.ctr[1 + 1], S.bctr[0]);
+        atomicAdd(&a.ctr[5 + 1], S.bctr[1]);
+        if (S.bctr[2]) {
+            atomicAdd(&a.ctr[0], S.bctr[2]);
+            atomicAdd(&a.ctr[9 + 1], S.bctr[2]);
+            atomicAdd(&a.ctr[13 + 1], S.bctr[3]);
+        }
+    }
+}
+
+// tile construction: degree of every bin entry; tiles of ~kTileE first edges
+__global__ void k_bin_entry_degrees(const int64_t *offsets, const int32_t *list, int64_t n, int64_t *deg) {
+    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k < n) deg[k] = offsets[list[k] + 1] - offsets[list[k]];
+    if (k == n) deg[k] = 0;
+}
+// coarse tile t starts at the first entry whose first edge is >= t*kTileE;
+// count of sub-tiles of <= kTileV entries per coarse tile
+__global__ void k_tile_coarse(const int64_t *pfx, int64_t n, int64_t ncoarse, int64_t *ks, int64_t *nsub) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t > ncoarse) return;
+    int64_t lo = 0, hi = n;                      // first k in [0, n] with pfx[k] >= t*E
+    const int64_t target = t * kTileE;
+    if (t == ncoarse) {
+        lo = n;
+    } else {
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (pfx[mid] < target) lo = mid + 1; else hi = mid;
+        }
+    }
+    ks[t] = lo;
+}
+__global__ void k_tile_count(const int64_t *ks, int64_t ncoarse, int64_t *nsub) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < ncoarse) nsub[t] = (ks[t + 1] - ks[t] + kTileV - 1) / kTileV;
+    if (t == ncoarse) nsub[t] = 0;
+}
+__global__ void k_tile_emit(const int64_t *ks, const int64_t *nsub_pfx, int64_t ncoarse, int64_t n, int32_t *tile_start) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < ncoarse) {
+        const int64_t b = nsub_pfx[t], e = nsub_pfx[t + 1];
+        for (int64_t q = b; q < e; ++q) tile_start[q] = (int32_t)(ks[t] + (q - b) * kTileV);
+    }
+    if (t == ncoarse) tile_start[nsub_pfx[ncoarse]] = (int32_t)n;
+}
+
+// ---------------------------------------------------------------------------
+// block-per-vertex kernel: one CTA per vertex, table (p1 <= 4095) in dynamic
+// shared memory, persistent grid-stride over the bin.  PAPER.md:243.
+// ---------------------------------------------------------------------------
+template <bool SYNC, bool W>
+__global__ void __launch_bounds__(kBlockThreads) k_block(SweepArgs a, const int32_t *__restrict__ list,
+                                                         int64_t n) {
+    extern __shared__ int32_t dyn[];
+    int32_t *Hk = dyn;
+    float *Hv = reinterpret_cast<float *>(dyn + kBlockCap);
+    __shared__ uint64_t red[kBlockThreads / 32];
+    __shared__ int s_act;
+    __shared__ int s_changed;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int s = threadIdx.x; s < kBlockCap; s += kBlockThreads) {
+        Hk[s] = kEmpty;
+        Hv[s] = 0.0f;
+    }
+    unsigned long long n_act = 0, n_edges = 0, n_changed = 0, n_changed_edges = 0;
+    __syncthreads();
+    for (int64_t t = blockIdx.x; t < n; t += gridDim.x) {
+        int32_t r = list[t];
+        int64_t v = r + a.row_begin;
+        if (threadIdx.x == 0) {
+            int f = a.flag_in[v];
+            s_act = f;
+            if (f && !SYNC) a.flag_in[v] = 0;
+        }
+        __syncthreads();
+        if (s_act) {
+            int64_t o = a.offsets[r];
+            uint32_t deg = (uint32_t)(a.offsets[r + 1] - o);
+            Hash h;
+            h.init(deg);
+            for (uint32_t b = (uint32_t)wid * 32; b < deg; b += kBlockThreads) {
+                int32_t key = kEmpty;
+                float w = 0.0f;
+                if (b + lane < deg) {
+                    const int32_t j = a.indices[o + b + lane];
+                    if (j != (int32_t)v) {
+                        key = a.lab_in[j];
+                        if (W) w = a.weights[o + b + lane];
+                    }
+                }
+                warp_batch_accumulate_atomic<W>(Hk, Hv, h, key, w);
+            }
+            __syncthreads();
+            TieOrder to;
+            to.init(a.tie_rule, h);
+            uint64_t best = 0;
+            for (uint32_t s = threadIdx.x; s < h.p1; s += kBlockThreads) {
+                int32_t k = Hk[s];
+                if (k != kEmpty) {
+                    uint64_t c = pack_cand(Hv[s], k, to);
+                    best = c > best ? c : best;
+                    Hk[s] = kEmpty;
+                    Hv[s] = 0.0f;
+                }
+            }
+            best = warp_max_u64(best);
+            if (lane == 0) red[wid] = best;
+            __syncthreads();
+            if (wid == 0) {
+                uint64_t b = lane < kBlockThreads / 32 ? red[lane] : 0;
+                b = warp_max_u64(b);
+                if (lane == 0) {
+                    int32_t ci = a.lab_in[v];
+                    int32_t cs = b ? cand_label(b, to) : kEmpty;
+                    int ch = accept_move(cs, ci, a.pickless);
+                    if (ch) a.lab_out[v] = cs;
+                    s_changed = ch;
+                    n_act += 1;
+                    n_edges += deg;
+                    n_changed += ch;
+                    n_changed_edges += ch ? deg : 0;
+                }
+            }
+            __syncthreads();
+            if (s_changed)
+                for (int64_t e = o + threadIdx.x; e < o + deg; e += kBlockThreads) a.flag_out[a.indices[e]] = 1;
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0 && n_act) {
+        atomicAdd(&a.ctr[1 + 2], n_act);
+        atomicAdd(&a.ctr[5 + 2], n_edges);
+        if (n_changed) {
+            atomicAdd(&a.ctr[0], n_changed);
+            atomicAdd(&a.ctr[9 + 2], n_changed);
+            atomicAdd(&a.ctr[13 + 2], n_changed_edges);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// giant vertices (degree >= giant_degree): the row is cut into chunks of
+// kGiantChunk edges, one CTA per chunk.  Each CTA pre-aggregates its chunk in
+// a shared-memory table, then folds the distinct (label, weight) pairs into
+// the vertex's GLOBAL-memory table (p1 = nextPow2(D)-1 slots),
+// recording newly claimed slots in an occupied list so the max-reduce and the
+// clear touch only occupied slots.
+// ---------------------------------------------------------------------------
+struct GiantArgs {
+    const int32_t *verts;        // [ng] local row ids
+    const int32_t *chunk_g;      // [nc] giant index of the chunk
+    const int64_t *chunk_e0;     // [nc] first edge of the chunk
+    const int64_t *chunk_e1;     // [nc] end edge of the chunk
+    const int64_t *table_off;    // [ng] first slot of the vertex's global table
+    int32_t *keys;               // global tables
+    float *vals;
+    int32_t *occ;                // occupied-slot lists (same offsets)
+    int32_t *occ_n;              // [ng]
+    uint8_t *active;             // [ng]
+    uint8_t *changed;            // [ng]
+};
+
+template <bool SYNC>
+__global__ void k_giant_snapshot(SweepArgs a, GiantArgs g, int64_t ng) {
+    int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= ng) return;
+    int64_t v = g.verts[k] + a.row_begin;
+    uint8_t f = a.flag_in[v];
+    g.active[k] = f ? 1 : 0;
+    g.changed[k] = 0;
+    if (!SYNC && f) a.flag_in[v] = 0;
+}
+
+template <bool SYNC, bool W>
+__global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a, GiantArgs g) {
+    extern __shared__ int32_t dyn[];
+    int32_t *Hk = dyn;
+    float *Hv = reinterpret_cast<float *>(dyn + kGiantCap);
+    const int64_t c = blockIdx.x;
+    const int32_t gi = g.chunk_g[c];
+    if (!g.active[gi]) return;
+    const int32_t r = g.verts[gi];
+    const int64_t v = r + a.row_begin;
+    const int64_t e0 = g.chunk_e0[c], e1 = g.chunk_e1[c];
+    for (int s = threadIdx.x; s < kGiantCap; s += kBlockThreads) {
+        Hk[s] = kEmpty;
+        Hv[s] = 0.0f;
+    }
+    __syncthreads();
+    Hash hc;
+    hc.init((uint32_t)(e1 - e0));
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int64_t b = e0 + wid * 32; b < e1; b += kBlockThreads) {
+        int32_t key = kEmpty;
+        float w = 0.0f;
+        if (b + lane < e1) {
+            const int32_t j = a.indices[b + lane];
+            if (j != (int32_t)v) {
+                key = a.lab_in[j];
+                if (W) w = a.weights[b + lane];
+            }
+        }
+        warp_batch_accumulate_atomic<W>(Hk, Hv, hc, key, w);
+    }
+    __syncthreads();
+    Hash hg;
+    hg.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
+    int32_t *gk = g.keys + g.table_off[gi];
+    float *gv = g.vals + g.table_off[gi];
+    int32_t *occ = g.occ + g.table_off[gi];
+    for (uint32_t s = threadIdx.x; s < hc.p1; s += kBlockThreads) {
+        int32_t k = Hk[s];
+        if (k != kEmpty) {
+            uint32_t slot;
+            if (ht_accumulate(gk, gv, hg, k, Hv[s], &slot)) occ[atomicAdd(&g.occ_n[gi], 1)] = (int32_t)slot;
+        }
+    }
+    if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
+}
+
+template <bool SYNC>
+__global__ void __launch_bounds__(kBlockThreads) k_giant_finalize(SweepArgs a, GiantArgs g) {
+    const int64_t gi = blockIdx.x;
+    if (!g.active[gi]) return;
+    __shared__ uint64_t red[kBlockThreads / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int32_t *gk = g.keys + g.table_off[gi];
+    float *gv = g.vals + g.table_off[gi];
+    const int32_t *occ = g.occ + g.table_off[gi];
+    const int32_t cnt = g.occ_n[gi];
+    const int32_t r = g.verts[gi];
+    Hash h;
+    h.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
+    TieOrder to;
+    to.init(a.tie_rule, h);
+    uint64_t best = 0;
+    for (int32_t q = threadIdx.x; q < cnt; q += kBlockThreads) {
+        int32_t s = occ[q];
+        uint64_t c = pack_cand(gv[s], gk[s], to);
+        best = c > best ? c : best;
+        gk[s] = kEmpty;
+        gv[s] = 0.0f;
+    }
+    best = warp_max_u64(best);
+    if (lane == 0) red[wid] = best;
+    __syncthreads();
+    if (wid == 0) {
+        uint64_t b = lane < kBlockThreads / 32 ? red[lane] : 0;
+        b = warp_max_u64(b);
+        if (lane == 0) {
+            g.occ_n[gi] = 0;
+            int64_t v = g.verts[gi] + a.row_begin;
+            int32_t ci = a.lab_in[v];
+            int32_t cs = b ? cand_label(b, to) : kEmpty;
+            bool ch = accept_move(cs, ci, a.pickless);
+            if (ch) {
+                a.lab_out[v] = cs;
+                g.changed[gi] = 1;
+                atomicAdd(&a.ctr[0], 1ull);
+                atomicAdd(&a.ctr[9 + 3], 1ull);
+                atomicAdd(&a.ctr[13 + 3], (unsigned long long)(a.offsets[r + 1] - a.offsets[r]));
+            }
+            atomicAdd(&a.ctr[1 + 3], 1ull);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kBlockThreads) k_giant_mark(SweepArgs a, GiantArgs g) {
+    const int64_t c = blockIdx.x;
+    const int32_t gi = g.chunk_g[c];
+    if (!g.changed[gi]) return;
+    for (int64_t e = g.chunk_e0[c] + threadIdx.x; e < g.chunk_e1[c]; e += kBlockThreads)
+        a.flag_out[a.indices[e]] = 1;
+}
+
+// ---------------------------------------------------------------------------
+// state / binning kernels
+// ---------------------------------------------------------------------------
+__global__ void k_init_state(int32_t *labels, uint8_t *flags, int64_t n) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        labels[i] = (int32_t)i;     // C <- [0 .. |V|)
+        flags[i] = 1;               // all vertices unprocessed
+    }
+}
+
+constexpr int kBinTile = 256;       // rows per tile (one per thread)
+constexpr int kBinTiles = 4;        // tiles per CTA
+
+__device__ __forceinline__ int bin_of(int64_t d, int32_t t1, int32_t t2, int32_t t3) {
+    return d == 0 ? -1 : d < t1 ? 0 : d < t2 ? 1 : d < t3 ? 2 : 3;
+}
+
+__global__ void __launch_bounds__(kBinTile) k_bin_count(const int64_t *offsets, int64_t n, int32_t t1, int32_t t2,
+                                                        int32_t t3, int64_t *counts, unsigned long long *edges) {
+    __shared__ int64_t c[4];
+    __shared__ unsigned long long ed[4];
+    if (threadIdx.x < 4) {
+        c[threadIdx.x] = 0;
+        ed[threadIdx.x] = 0;
+    }
+    __syncthreads();
+    for (int k = 0; k < kBinTiles; ++k) {
+        int64_t r = ((int64_t)blockIdx.x * kBinTiles + k) * kBinTile + threadIdx.x;
+        if (r < n) {
+            int64_t d = offsets[r + 1] - offsets[r];
+            int b = bin_of(d, t1, t2, t3);
+            if (b >= 0) {
+                atomicAdd((unsigned long long *)&c[b], 1ull);
+                atomicAdd(&ed[b], (unsigned long long)d);
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x < 4) {
+        counts[(int64_t)blockIdx.x * 4 + threadIdx.x] = c[threadIdx.x];
+        atomicAdd(&edges[threadIdx.x], ed[threadIdx.x]);
+    }
+}
+
+// exclusive scan of counts[nb][4] per bin (single CTA of 1024 threads)
+__global__ void __launch_bounds__(1024) k_bin_scan(int64_t *counts, int64_t nb, int64_t *totals) {
+    __shared__ int64_t ws[32];
+    __shared__ int64_t carry_s;
+    for (int b = 0; b < 4; ++b) {
+        if (threadIdx.x == 0) carry_s = 0;
+        __syncthreads();
+        for (int64_t base = 0; base < nb; base += 1024) {
+            int64_t i = base + threadIdx.x;
+            int64_t x = i < nb ? counts[i * 4 + b] : 0;
+            // inclusive warp scan
+            int64_t y = x;
+            for (int o = 1; o < 32; o <<= 1) {
+                int64_t z = __shfl_up_sync(0xFFFFFFFFu, y, o);
+                if ((threadIdx.x & 31) >= o) y += z;
+            }
+            if ((threadIdx.x & 31) == 31) ws[threadIdx.x >> 5] = y;
+            __syncthreads();
+            if (threadIdx.x < 32) {
+                int64_t s = ws[threadIdx.x];
+                for (int o = 1; o < 32; o <<= 1) {
+                    int64_t z = __shfl_up_sync(0xFFFFFFFFu, s, o);
+                    if (threadIdx.x >= o) s += z;
+                }
+                ws[threadIdx.x] = s;
+            }
+            __syncthreads();
+            int64_t warp_prefix = (threadIdx.x >> 5) ? ws[(threadIdx.x >> 5) - 1] : 0;
+            int64_t carry = carry_s;
+            if (i < nb) counts[i * 4 + b] = carry + warp_prefix + y - x;
+            __syncthreads();
+            if (threadIdx.x == 1023) carry_s = carry + warp_prefix + y;
+            __syncthreads();
+        }
+        if (threadIdx.x == 0) totals[b] = carry_s;
+        __syncthreads();
+    }
+}
+
+struct BinLists {
+    int32_t *l[4];
+};
+
+__global__ void __launch_bounds__(kBinTile) k_bin_scatter(const int64_t *offsets, int64_t n, int32_t t1, int32_t t2,
+                                                          int32_t t3, const int64_t *base, BinLists lists) {
+    __shared__ int32_t wc[kBinTile / 32][4];
+    __shared__ int64_t run[4];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (threadIdx.x < 4) run[threadIdx.x] = base[(int64_t)blockIdx.x * 4 + threadIdx.x];
+    __syncthreads();
+    for (int k = 0; k < kBinTiles; ++k) {
+        int64_t r = ((int64_t)blockIdx.x * kBinTiles + k) * kBinTile + threadIdx.x;
+        int b = -1;
+        if (r < n) b = bin_of(offsets[r + 1] - offsets[r], t1, t2, t3);
+        unsigned lt = (1u << lane) - 1;
+        int my_rank = 0;
+        for (int q = 0; q < 4; ++q) {
+            unsigned m = __ballot_sync(0xFFFFFFFFu, b == q);
+            if (b == q) my_rank = __popc(m & lt);
+            if (lane == 0) wc[wid][q] = __popc(m);
+        }
+        __syncthreads();
+        if (b >= 0) {
+            int64_t off = run[b];
+            for (int w = 0; w < wid; ++w) off += wc[w][b];
+            lists.l[b][off + my_rank] = (int32_t)r;
+        }
+        __syncthreads();
+        if (threadIdx.x < 4) {
+            int64_t s = 0;
+            for (int w = 0; w < kBinTile / 32; ++w) s += wc[w][threadIdx.x];
+            run[threadIdx.x] += s;
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void k_gather_degrees(const int64_t *offsets, const int32_t *rows, int64_t n, int64_t *out) {
+    int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (k < n) {
+        out[k] = offsets[rows[k] + 1] - offsets[rows[k]];
+        out[n + k] = offsets[rows[k]];
+    }
+}
+
+// ---------------------------------------------------------------------------
+// modularity (Eq. 1, second form, R11), float64
+// ---------------------------------------------------------------------------
+// acc[0] += sigma_intra, acc[1] += 2m; Sigma[c] += K_i
+template <bool W>
+__global__ void __launch_bounds__(256) k_mod_rows(const int64_t *__restrict__ offsets, const int32_t *__restrict__ indices,
+                                                  const float *__restrict__ weights, const int32_t *__restrict__ labels,
+                                                  int64_t n_rows, int64_t row_begin, double *Sigma, double *acc) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+    double intra = 0.0, tot = 0.0;
+    for (int64_t r = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); r < n_rows; r += nw) {
+        int64_t v = r + row_begin;
+        int32_t cv = labels[v];
+        double K = 0.0, in = 0.0;
+        for (int64_t e = offsets[r] + lane; e < offsets[r + 1]; e += 32) {
+            double w = W ? (double)weights[e] : 1.0;
+            K += w;
+            if (labels[indices[e]] == cv) in += w;
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            K += __shfl_xor_sync(0xFFFFFFFFu, K, o);
+            in += __shfl_xor_sync(0xFFFFFFFFu, in, o);
+        }
+        if (lane == 0) {
+            if (K != 0.0) atomicAdd(&Sigma[cv], K);
+            intra += in;
+            tot += K;
+        }
+    }
+    __shared__ double s_in[8], s_tot[8];
+    if (lane == 0) {
+        s_in[threadIdx.x >> 5] = intra;
+        s_tot[threadIdx.x >> 5] = tot;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double a = 0, b = 0;
+        for (int w = 0; w < (int)(blockDim.x / 32); ++w) {
+            a += s_in[w];
+            b += s_tot[w];
+        }
+        atomicAdd(&acc[0], a);
+        atomicAdd(&acc[1], b);
+    }
+}
+
+// acc[2] += sum_c Sigma_c^2 ; Sigma reset to 0 when `clear`
+__global__ void __launch_bounds__(256) k_mod_finish(double *Sigma, int64_t n, double *acc, int clear) {
+    double s = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        double x = Sigma[i];
+        s += x * x;
+        if (clear) Sigma[i] = 0.0;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xFFFFFFFFu, s, o);
+    __shared__ double ws[8];
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0;
+        for (int w = 0; w < (int)(blockDim.x / 32); ++w) t += ws[w];
+        atomicAdd(&acc[2], t);
+    }
+}
+
+int num_sms() {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    return sms;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// handle
+// ---------------------------------------------------------------------------
+struct nulpa_graph {
+    int64_t n_rows = 0, n_global = 0, row_begin = 0, M = 0;
+    int64_t *offsets = nullptr;
+    int32_t *indices = nullptr;
+    float *weights = nullptr;
+    bool own_csr = false;
+    int32_t *labels = nullptr;      // current labels (own or bound)
+    uint8_t *flags = nullptr;       // current flags (own or bound)
+    int32_t *own_labels = nullptr;
+    uint8_t *own_flags = nullptr;
+    int32_t *labels_prev = nullptr; // sync-mode snapshot
+    uint8_t *flags_prev = nullptr;
+    cudaStream_t stream = nullptr;
+    // bins
+    int32_t t1 = 0, t2 = 0, t3 = 0;
+    bool bins_built = false;
+    int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
+    int64_t bin_n[4] = {0, 0, 0, 0};
+    int64_t bin_e[4] = {0, 0, 0, 0};
+    // giant
+    int64_t n_chunks = 0;
+    int32_t *chunk_g = nullptr;
+    int64_t *chunk_e0 = nullptr, *chunk_e1 = nullptr, *table_off = nullptr;
+    int32_t *gkeys = nullptr, *occ = nullptr, *occ_n = nullptr;
+    float *gvals = nullptr;
+    uint8_t *gactive = nullptr, *gchanged = nullptr;
+    // tiles of the warp bin
+    int64_t n_tiles = 0;
+    int32_t *tile_start = nullptr;
+    int warp_kernel = 0;                     // 0: k_tile, 1: k_warp (env NULPA_WARP_KERNEL)
+    // counters
+    unsigned long long *ctr = nullptr;       // device [kMaxIter+1][kCtr]
+    unsigned long long *ctr_host = nullptr;  // pinned
+    int sweep_slot = 0;                      // counter slot used by nulpa_sweep
+    // modularity scratch
+    double *Sigma = nullptr;
+    double *macc = nullptr;
+    // timing
+    cudaEvent_t ev[2 * 4 * (kMaxIter + 1)];
+    cudaEvent_t ev_run[2];
+    bool events = false;
+    nulpa_stats stats;
+};
+
+namespace {
+
+template <typename T>
+int dalloc(T **p, size_t n) {
+    if (n == 0) n = 1;
+    cudaError_t e = cudaMalloc((void **)p, n * sizeof(T));
+    if (e != cudaSuccess) {
+        *p = nullptr;
+        return fail(NULPA_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", n * sizeof(T), cudaGetErrorString(e));
+    }
+    return NULPA_OK;
+}
+
+void free_bins(nulpa_graph *g) {
+    for (int b = 0; b < 4; ++b) {
+        cudaFree(g->bin_list[b]);
+        g->bin_list[b] = nullptr;
+        g->bin_n[b] = g->bin_e[b] = 0;
+    }
+    cudaFree(g->chunk_g);
+    cudaFree(g->chunk_e0);
+    cudaFree(g->chunk_e1);
+    cudaFree(g->table_off);
+    cudaFree(g->gkeys);
+    cudaFree(g->gvals);
+    cudaFree(g->occ);
+    cudaFree(g->occ_n);
+    cudaFree(g->gactive);
+    cudaFree(g->gchanged);
+    cudaFree(g->tile_start);
+    g->tile_start = nullptr;
+    g->n_tiles = 0;
+    g->chunk_g = nullptr;
+    g->chunk_e0 = g->chunk_e1 = g->table_off = nullptr;
+    g->gkeys = g->occ = g->occ_n = nullptr;
+    g->gvals = nullptr;
+    g->gactive = g->gchanged = nullptr;
+    g->n_chunks = 0;
+    g->bins_built = false;
+}
+
+__global__ void k_fill_i32(int32_t *p, int64_t n, int32_t v) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+
+int grid_for(int64_t n, int threads, int cap_blocks = 0) {
+    int64_t b = (n + threads - 1) / threads;
+    if (cap_blocks > 0 && b > cap_blocks) b = cap_blocks;
+    return (int)std::max<int64_t>(b, 1);
+}
+
+// Row a1: the degree-binned frontier.
+int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
+    free_bins(g);
+    g->t1 = t1;
+    g->t2 = t2;
+    g->t3 = t3;
+    const int64_t n = g->n_rows;
+    const int64_t per = (int64_t)kBinTile * kBinTiles;
+    const int64_t nb = (n + per - 1) / per;
+    int64_t *counts = nullptr, *totals = nullptr;
+    unsigned long long *edges = nullptr;
+    CHECK(dalloc(&counts, (size_t)std::max<int64_t>(nb, 1) * 4));
+    CHECK(dalloc(&totals, 4));
+    CHECK(dalloc(&edges, 4));
+    CU(cudaMemsetAsync(edges, 0, 4 * sizeof(unsigned long long), g->stream));
+    if (nb > 0) {
+        k_bin_count<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, edges);
+        CU(cudaGetLastError());
+        k_bin_scan<<<1, 1024, 0, g->stream>>>(counts, nb, totals);
+        CU(cudaGetLastError());
+    } else {
+        CU(cudaMemsetAsync(totals, 0, 4 * sizeof(int64_t), g->stream));
+    }
+    int64_t ht[4];
+    unsigned long long he[4];
+    CU(cudaMemcpyAsync(ht, totals, sizeof ht, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaMemcpyAsync(he, edges, sizeof he, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    BinLists L;
+    for (int b = 0; b < 4; ++b) {
+        g->bin_n[b] = ht[b];
+        g->bin_e[b] = (int64_t)he[b];
+        CHECK(dalloc(&g->bin_list[b], (size_t)ht[b]));
+        L.l[b] = g->bin_list[b];
+    }
+    if (nb > 0) {
+        k_bin_scatter<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, L);
+        CU(cudaGetLastError());
+    }
+    // tiles of the warp bin (k_tile)
+    if (g->bin_n[1] > 0) {
+        const int64_t n1 = g->bin_n[1];
+        int64_t *deg1 = nullptr, *pfx1 = nullptr;
+        CHECK(dalloc(&deg1, (size_t)n1 + 1));
+        CHECK(dalloc(&pfx1, (size_t)n1 + 1));
+        k_bin_entry_degrees<<<grid_for(n1 + 1, 256), 256, 0, g->stream>>>(g->offsets, g->bin_list[1], n1, deg1);
+        CU(cudaGetLastError());
+        size_t tmp_bytes = 0;
+        CU(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, deg1, pfx1, n1 + 1, g->stream));
+        void *tmp = nullptr;
+        CU(cudaMalloc(&tmp, tmp_bytes));
+        CU(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, deg1, pfx1, n1 + 1, g->stream));
+        int64_t E1 = 0;
+        CU(cudaMemcpyAsync(&E1, pfx1 + n1, sizeof E1, cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        const int64_t ncoarse = (E1 + kTileE - 1) / kTileE;
+        int64_t *ks = nullptr, *nsub = nullptr, *nsub_pfx = nullptr;
+        CHECK(dalloc(&ks, (size_t)ncoarse + 1));
+        CHECK(dalloc(&nsub, (size_t)ncoarse + 1));
+        CHECK(dalloc(&nsub_pfx, (size_t)ncoarse + 1));
+        k_tile_coarse<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(pfx1, n1, ncoarse, ks, nsub);
+        k_tile_count<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(ks, ncoarse, nsub);
+        CU(cudaGetLastError());
+        size_t tmp2 = 0;
+        CU(cub::DeviceScan::ExclusiveSum(nullptr, tmp2, nsub, nsub_pfx, ncoarse + 1, g->stream));
+        if (tmp2 > tmp_bytes) {
+            cudaFree(tmp);
+            CU(cudaMalloc(&tmp, tmp2));
+            tmp_bytes = tmp2;
+        }
+        CU(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, nsub, nsub_pfx, ncoarse + 1, g->stream));
+        int64_t nt = 0;
+        CU(cudaMemcpyAsync(&nt, nsub_pfx + ncoarse, sizeof nt, cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        g->n_tiles = nt;
+        CHECK(dalloc(&g->tile_start, (size_t)nt + 1));
+        k_tile_emit<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(ks, nsub_pfx, ncoarse, n1, g->tile_start);
+        CU(cudaGetLastError());
+        CU(cudaStreamSynchronize(g->stream));
+        cudaFree(tmp);
+        cudaFree(deg1);
+        cudaFree(pfx1);
+        cudaFree(ks);
+        cudaFree(nsub);
+        cudaFree(nsub_pfx);
+    }
+    // giant chunks (host-side bookkeeping over the few giant vertices)
+    const int64_t ng = g->bin_n[3];
+    if (ng > 0) {
+        int64_t *ddeg = nullptr;
+        CHECK(dalloc(&ddeg, (size_t)(2 * ng)));   // [degrees | row offsets]
+        k_gather_degrees<<<grid_for(ng, 256), 256, 0, g->stream>>>(g->offsets, g->bin_list[3], ng, ddeg);
+        CU(cudaGetLastError());
+        std::vector<int64_t> deg(ng);
+        std::vector<int32_t> rows(ng);
+        CU(cudaMemcpyAsync(deg.data(), ddeg, ng * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaMemcpyAsync(rows.data(), g->bin_list[3], ng * sizeof(int32_t), cudaMemcpyDeviceToHost, g->stream));
+        std::vector<int64_t> roff(ng);
+        CU(cudaMemcpyAsync(roff.data(), ddeg + ng, ng * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        cudaFree(ddeg);
+        std::vector<int32_t> cg;
+        std::vector<int64_t> c0, c1, toff(ng);
+        int64_t slots = 0;
+        for (int64_t k = 0; k < ng; ++k) {
+            toff[k] = slots;
+            slots += capacity_p1((uint32_t)deg[k]) + 1;
+            for (int64_t e = 0; e < deg[k]; e += kGiantChunk) {
+                cg.push_back((int32_t)k);
+                c0.push_back(roff[k] + e);
+                c1.push_back(roff[k] + std::min<int64_t>(deg[k], e + kGiantChunk));
+            }
+        }
+        g->n_chunks = (int64_t)cg.size();
+        CHECK(dalloc(&g->chunk_g, cg.size()));
+        CHECK(dalloc(&g->chunk_e0, c0.size()));
+        CHECK(dalloc(&g->chunk_e1, c1.size()));
+        CHECK(dalloc(&g->table_off, (size_t)ng));
+        CHECK(dalloc(&g->gkeys, (size_t)slots));
+        CHECK(dalloc(&g->gvals, (size_t)slots));
+        CHECK(dalloc(&g->occ, (size_t)slots));
+        CHECK(dalloc(&g->occ_n, (size_t)ng));
+        CHECK(dalloc(&g->gactive, (size_t)ng));
+        CHECK(dalloc(&g->gchanged, (size_t)ng));
+        CU(cudaMemcpy(g->chunk_g, cg.data(), cg.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(g->chunk_e0, c0.data(), c0.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(g->chunk_e1, c1.data(), c1.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(g->table_off, toff.data(), toff.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+        k_fill_i32<<<grid_for(slots, 256, 4096), 256, 0, g->stream>>>(g->gkeys, slots, kEmpty);
+        CU(cudaGetLastError());
+        CU(cudaMemsetAsync(g->gvals, 0, slots * sizeof(float), g->stream));
+        CU(cudaMemsetAsync(g->occ_n, 0, ng * sizeof(int32_t), g->stream));
+    }
+    CU(cudaStreamSynchronize(g->stream));
+    cudaFree(counts);
+    cudaFree(totals);
+    cudaFree(edges);
+    for (int b = 0; b < 4; ++b) {
+        g->stats.bin_vertices[b] = g->bin_n[b];
+        g->stats.bin_edges[b] = g->bin_e[b];
+    }
+    g->bins_built = true;
+    return NULPA_OK;
+}
+
+int validate_params(const nulpa_params &p) {
+    if (!(p.tolerance >= 0.0)) return fail(NULPA_EINVAL, "tolerance must be >= 0");
+    if (p.max_iterations < 0) return fail(NULPA_EINVAL, "max_iterations must be >= 0");
+    if (p.mode != NULPA_ASYNC && p.mode != NULPA_SYNC) return fail(NULPA_EINVAL, "mode must be NULPA_ASYNC or NULPA_SYNC");
+    if (p.switch_degree < 1 || p.switch_degree > 33)
+        return fail(NULPA_EINVAL, "switch_degree must be in [1, 33] (thread-per-vertex tables live in registers)");
+    if (p.block_degree < p.switch_degree || p.block_degree > 256)
+        return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
+    if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
+    if (p.bin_order != 0 && p.bin_order != 1) return fail(NULPA_EINVAL, "bin_order must be 0 or 1");
+    if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
+        return fail(NULPA_EINVAL, "giant_degree must be in [block_degree, 4096] (CTA tables hold 4095 slots)");
+    return NULPA_OK;
+}
+
+int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
+    if (g->bins_built && g->t1 == p.switch_degree && g->t2 == p.block_degree && g->t3 == p.giant_degree) return NULPA_OK;
+    return build_bins(g, p.switch_degree, p.block_degree, p.giant_degree);
+}
+
+template <bool SYNC, bool W>
+int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
+    const int64_t n = g->bin_n[0];
+    const int grid = grid_for(n, kThreadThreads);
+    if (g->t1 <= 5)
+        k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+    else if (g->t1 <= 9)
+        k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+    else if (g->t1 <= 17)
+        k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+    else
+        k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+    CU(cudaGetLastError());
+    return NULPA_OK;
+}
+
+template <bool SYNC, bool W>
+int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
+    SweepArgs a;
+    a.tie_rule = p.tie_rule;
+    a.offsets = g->offsets;
+    a.indices = g->indices;
+    a.weights = g->weights;
+    a.row_begin = g->row_begin;
+    a.pickless = pickless;
+    a.ctr = ctr;
+    if (SYNC) {
+        CU(cudaMemcpyAsync(g->labels_prev, g->labels, g->n_global * sizeof(int32_t), cudaMemcpyDeviceToDevice, g->stream));
+        CU(cudaMemcpyAsync(g->flags_prev, g->flags, g->n_global, cudaMemcpyDeviceToDevice, g->stream));
+        CU(cudaMemsetAsync(g->flags, 0, g->n_global, g->stream));
+        a.lab_in = g->labels_prev;
+        a.flag_in = g->flags_prev;
+        g->stats.other_launches += 3;
+    } else {
+        a.lab_in = g->labels;
+        a.flag_in = g->flags;
+    }
+    a.lab_out = g->labels;
+    a.flag_out = g->flags;
+    const int sms = num_sms();
+    auto rec = [&](int b, int which) -> int {
+        if (timing) CU(cudaEventRecord(g->ev[(slot * 4 + b) * 2 + which], g->stream));
+        return NULPA_OK;
+    };
+    auto run_giant = [&]() -> int {
+        const int64_t ng = g->bin_n[3];
+        CHECK(rec(3, 0));
+        if (ng > 0) {
+            GiantArgs ga;
+            ga.verts = g->bin_list[3];
+            ga.chunk_g = g->chunk_g;
+            ga.chunk_e0 = g->chunk_e0;
+            ga.chunk_e1 = g->chunk_e1;
+            ga.table_off = g->table_off;
+            ga.keys = g->gkeys;
+            ga.vals = g->gvals;
+            ga.occ = g->occ;
+            ga.occ_n = g->occ_n;
+            ga.active = g->gactive;
+            ga.changed = g->gchanged;
+            const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float));
+            static bool attr_set = false;   // one per template instantiation
+            if (!attr_set) {
+                CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                attr_set = true;
+            }
+            k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, g->stream>>>(a, ga, ng);
+            k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, g->stream>>>(a, ga);
+            k_giant_finalize<SYNC><<<(unsigned)ng, kBlockThreads, 0, g->stream>>>(a, ga);
+            k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
+            CU(cudaGetLastError());
+            g->stats.launches[3] += 4;
+        }
+        CHECK(rec(3, 1));
+        return NULPA_OK;
+    };
+    auto run_block = [&]() -> int {
+        const int64_t n = g->bin_n[2];
+        CHECK(rec(2, 0));
+        if (n > 0) {
+            const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
+            k_block<SYNC, W><<<grid_for(n, 1, sms * 4), kBlockThreads, smem, g->stream>>>(a, g->bin_list[2], n);
+            CU(cudaGetLastError());
+            g->stats.launches[2] += 1;
+        }
+        CHECK(rec(2, 1));
+        return NULPA_OK;
+    };
+    auto run_warp = [&]() -> int {
+        const int64_t n = g->bin_n[1];
+        CHECK(rec(1, 0));
+        if (n > 0) {
+            if (g->warp_kernel == 0) {
+                const size_t smem = sizeof(TileSmem<W>);
+                static bool attr_set = false;
+                if (!attr_set) {
+                    CU(cudaFuncSetAttribute(k_tile<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                    attr_set = true;
+                }
+                k_tile<SYNC, W><<<grid_for(g->n_tiles, 1, sms * 4), kTileThreads, smem, g->stream>>>(
+                    a, g->bin_list[1], g->tile_start, g->n_tiles);
+            } else {
+                k_warp<SYNC, W><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * 8), kWarpThreads, 0, g->stream>>>(a, g->bin_list[1], n);
+            }
+            CU(cudaGetLastError());
+            g->stats.launches[1] += 1;
+        }
+        CHECK(rec(1, 1));
+        return NULPA_OK;
+    };
+    auto run_thread = [&]() -> int {
+        const int64_t n = g->bin_n[0];
+        CHECK(rec(0, 0));
+        if (n > 0) {
+            CHECK((launch_thread_bin<SYNC, W>(g, a)));
+            g->stats.launches[0] += 1;
+        }
+        CHECK(rec(0, 1));
+        return NULPA_OK;
+    };
+    if (p.bin_order == 0) {
+        CHECK(run_giant());
+        CHECK(run_block());
+        CHECK(run_warp());
+        CHECK(run_thread());
+    } else {
+        CHECK(run_thread());
+        CHECK(run_warp());
+        CHECK(run_block());
+        CHECK(run_giant());
+    }
+    return NULPA_OK;
+}
+
+int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
+    const bool w = g->weights != nullptr;
+    if (p.mode == NULPA_SYNC) {
+        if (!g->labels_prev) {
+            CHECK(dalloc(&g->labels_prev, (size_t)g->n_global));
+            CHECK(dalloc(&g->flags_prev, (size_t)g->n_global));
+        }
+        return w ? sweep_impl<true, true>(g, pickless, p, ctr, timing, slot) : sweep_impl<true, false>(g, pickless, p, ctr, timing, slot);
+    }
+    return w ? sweep_impl<false, true>(g, pickless, p, ctr, timing, slot) : sweep_impl<false, false>(g, pickless, p, ctr, timing, slot);
+}
+
+int reset_state(nulpa_graph *g) {
+    k_init_state<<<grid_for(g->n_global, 256, num_sms() * 16), 256, 0, g->stream>>>(g->labels, g->flags, g->n_global);
+    CU(cudaGetLastError());
+    g->stats.other_launches += 1;
+    return NULPA_OK;
+}
+
+void zero_stats_counts(nulpa_stats *s) {
+    int64_t bv[4], be[4];
+    memcpy(bv, s->bin_vertices, sizeof bv);
+    memcpy(be, s->bin_edges, sizeof be);
+    memset(s, 0, sizeof *s);
+    memcpy(s->bin_vertices, bv, sizeof bv);
+    memcpy(s->bin_edges, be, sizeof be);
+}
+
+int ensure_events(nulpa_graph *g) {
+    if (g->events) return NULPA_OK;
+    for (auto &e : g->ev) CU(cudaEventCreate(&e));
+    CU(cudaEventCreate(&g->ev_run[0]));
+    CU(cudaEventCreate(&g->ev_run[1]));
+    g->events = true;
+    return NULPA_OK;
+}
+
+int resolve_mem(const void *p, int memkind) {
+    if (memkind != NULPA_MEM_HOST && memkind != NULPA_MEM_DEVICE) return fail(NULPA_EINVAL, "memkind must be NULPA_MEM_HOST or NULPA_MEM_DEVICE");
+    (void)p;
+    return NULPA_OK;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------------------
+// C ABI
+// ---------------------------------------------------------------------------
+extern "C" {
+
+void nulpa_default_params(nulpa_params *p) {
+    if (!p) return;
+    p->tolerance = 0.05;
+    p->max_iterations = 20;
+    p->pickless_period = 4;
+    p->mode = NULPA_ASYNC;
+    p->switch_degree = 16;
+    p->block_degree = 256;
+    p->giant_degree = 4096;
+    p->reset = 1;
+    p->timing = 0;
+    p->tie_rule = NULPA_TIE_SMALLEST;
+    p->bin_order = 1;
+}
+
+const char *nulpa_last_error(void) { return g_err.c_str(); }
+
+const char *nulpa_version(void) { return "nulpa 0.1.0 sm_100a"; }
+
+int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *weights, int64_t n_rows,
+                 int64_t n_global, int64_t row_begin, int memkind, void *stream, nulpa_graph **out) {
+    g_err.clear();
+    if (!out) return fail(NULPA_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (!offsets) return fail(NULPA_EINVAL, "offsets is NULL");
+    if (n_rows < 0 || n_global < 0 || row_begin < 0 || row_begin + n_rows > n_global)
+        return fail(NULPA_EINVAL, "need 0 <= row_begin, row_begin + n_rows <= n_global");
+    if (n_global > INT32_MAX) return fail(NULPA_EINVAL, "n_global must fit int32 vertex IDs");
+    CHECK(resolve_mem(offsets, memkind));
+    nulpa_graph *g = new nulpa_graph();
+    memset(&g->stats, 0, sizeof g->stats);
+    if (const char *e = getenv("NULPA_WARP_KERNEL")) g->warp_kernel = atoi(e);
+    g->n_rows = n_rows;
+    g->n_global = n_global;
+    g->row_begin = row_begin;
+    g->stream = (cudaStream_t)stream;
+    auto bail = [&](int code) {
+        nulpa_destroy(g);
+        return code;
+    };
+    int64_t M = 0;
+    if (memkind == NULPA_MEM_HOST) {
+        M = offsets[n_rows];
+        if (offsets[0] != 0) return bail(fail(NULPA_EINVAL, "offsets[0] must be 0"));
+    } else {
+        int64_t o0 = 0;
+        cudaError_t e = cudaMemcpy(&M, offsets + n_rows, sizeof M, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(&o0, offsets, sizeof o0, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) return bail(fail(NULPA_ECUDA, "reading device offsets failed: %s", cudaGetErrorString(e)));
+        if (o0 != 0) return bail(fail(NULPA_EINVAL, "offsets[0] must be 0"));
+    }
+    if (M < 0) return bail(fail(NULPA_EINVAL, "offsets[n_rows] must be >= 0"));
+    if (M > 0 && !indices) return bail(fail(NULPA_EINVAL, "indices is NULL"));
+    g->M = M;
+    if (memkind == NULPA_MEM_DEVICE) {
+        g->offsets = const_cast<int64_t *>(offsets);
+        g->indices = const_cast<int32_t *>(indices);
+        g->weights = const_cast<float *>(weights);
+        g->own_csr = false;
+    } else {
+        g->own_csr = true;
+        int r;
+        if ((r = dalloc(&g->offsets, (size_t)n_rows + 1))) return bail(r);
+        if ((r = dalloc(&g->indices, (size_t)M))) return bail(r);
+        if (weights && (r = dalloc(&g->weights, (size_t)M))) return bail(r);
+        cudaError_t e = cudaMemcpyAsync(g->offsets, offsets, (n_rows + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream);
+        if (e == cudaSuccess && M) e = cudaMemcpyAsync(g->indices, indices, M * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream);
+        if (e == cudaSuccess && M && weights) e = cudaMemcpyAsync(g->weights, weights, M * sizeof(float), cudaMemcpyHostToDevice, g->stream);
+        if (e != cudaSuccess) return bail(fail(NULPA_ECUDA, "host->device copy failed: %s", cudaGetErrorString(e)));
+    }
+    int r;
+    if ((r = dalloc(&g->own_labels, (size_t)n_global))) return bail(r);
+    if ((r = dalloc(&g->own_flags, (size_t)n_global))) return bail(r);
+    g->labels = g->own_labels;
+    g->flags = g->own_flags;
+    if ((r = dalloc(&g->ctr, (size_t)(kMaxIter + 1) * kCtr))) return bail(r);
+    if (cudaMallocHost((void **)&g->ctr_host, (kMaxIter + 1) * kCtr * sizeof(unsigned long long)) != cudaSuccess)
+        return bail(fail(NULPA_ENOMEM, "cudaMallocHost failed"));
+    if ((r = reset_state(g))) return bail(r);
+    nulpa_params p;
+    nulpa_default_params(&p);
+    if ((r = build_bins(g, p.switch_degree, p.block_degree, p.giant_degree))) return bail(r);
+    *out = g;
+    return NULPA_OK;
+}
+
+int nulpa_bind_state(nulpa_graph *g, int32_t *labels_device, uint8_t *flags_device) {
+    if (!g || !labels_device || !flags_device) return fail(NULPA_EINVAL, "null argument");
+    g->labels = labels_device;
+    g->flags = flags_device;
+    return NULPA_OK;
+}
+
+int nulpa_reset(nulpa_graph *g) {
+    if (!g) return fail(NULPA_EINVAL, "null handle");
+    return reset_state(g);
+}
+
+int nulpa_sweep(nulpa_graph *g, int pickless, const nulpa_params *params, int64_t *changed) {
+    if (!g) return fail(NULPA_EINVAL, "null handle");
+    nulpa_params p;
+    if (params) p = *params; else nulpa_default_params(&p);
+    CHECK(validate_params(p));
+    CHECK(ensure_bins(g, p));
+    unsigned long long *ctr = g->ctr + (size_t)kMaxIter * kCtr;   // spare slot
+    CU(cudaMemsetAsync(ctr, 0, kCtr * sizeof(unsigned long long), g->stream));
+    CHECK(sweep(g, pickless ? 1 : 0, p, ctr, false, 0));
+    if (changed) {
+        CU(cudaMemcpyAsync(g->ctr_host, ctr, kCtr * sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        *changed = (int64_t)g->ctr_host[0];
+        for (int b = 0; b < 4; ++b) {
+            g->stats.vertices_processed[b] += (int64_t)g->ctr_host[1 + b];
+            g->stats.edges_scanned[b] += (int64_t)g->ctr_host[5 + b];
+            g->stats.vertices_changed[b] += (int64_t)g->ctr_host[9 + b];
+            g->stats.changed_edges[b] += (int64_t)g->ctr_host[13 + b];
+        }
+    }
+    return NULPA_OK;
+}
+
+int nulpa_run(nulpa_graph *g, const nulpa_params *params, nulpa_stats *stats) {
+    if (!g) return fail(NULPA_EINVAL, "null handle");
+    nulpa_params p;
+    if (params) p = *params; else nulpa_default_params(&p);
+    CHECK(validate_params(p));
+    CHECK(ensure_bins(g, p));
+    const int maxit = std::min(p.max_iterations, kMaxIter);
+    if (p.max_iterations > kMaxIter) return fail(NULPA_EINVAL, "max_iterations must be <= %d", kMaxIter);
+    zero_stats_counts(&g->stats);
+    CHECK(ensure_events(g));
+    const bool timing = p.timing != 0;
+    CU(cudaMemsetAsync(g->ctr, 0, (size_t)(kMaxIter + 1) * kCtr * sizeof(unsigned long long), g->stream));
+    CU(cudaEventRecord(g->ev_run[0], g->stream));
+    if (p.reset) CHECK(reset_state(g));
+    int l = 0;
+    int converged = 0;
+    for (; l < maxit; ++l) {
+        const int pl = p.pickless_period > 0 && (l % p.pickless_period) == 0;
+        unsigned long long *ctr = g->ctr + (size_t)l * kCtr;
+        CHECK(sweep(g, pl, p, ctr, timing, l));
+        CU(cudaMemcpyAsync(g->ctr_host + (size_t)l * kCtr, ctr, sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        const int64_t dn = (int64_t)g->ctr_host[(size_t)l * kCtr];
+        if (!pl && (double)dn / (double)g->n_global < p.tolerance) {
+            ++l;
+            converged = 1;
+            break;
+        }
+    }
+    CU(cudaEventRecord(g->ev_run[1], g->stream));
+    CU(cudaMemcpyAsync(g->ctr_host, g->ctr, (size_t)kMaxIter * kCtr * sizeof(unsigned long long), cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    nulpa_stats &s = g->stats;
+    s.iterations = l;
+    s.converged = converged;
+    for (int it = 0; it < l; ++it) {
+        const unsigned long long *c = g->ctr_host + (size_t)it * kCtr;
+        s.changed[it] = (int64_t)c[0];
+        for (int b = 0; b < 4; ++b) {
+            s.vertices_processed[b] += (int64_t)c[1 + b];
+            s.edges_scanned[b] += (int64_t)c[5 + b];
+            s.vertices_changed[b] += (int64_t)c[9 + b];
+            s.changed_edges[b] += (int64_t)c[13 + b];
+        }
+        if (timing) {
+            for (int b = 0; b < 4; ++b) {
+                float ms = 0;
+                CU(cudaEventElapsedTime(&ms, g->ev[(it * 4 + b) * 2], g->ev[(it * 4 + b) * 2 + 1]));
+                s.kernel_ms[b] += ms;
+            }
+        }
+    }
+    float rms = 0;
+    CU(cudaEventElapsedTime(&rms, g->ev_run[0], g->ev_run[1]));
+    s.run_ms = rms;
+    if (stats) *stats = s;
+    return NULPA_OK;
+}
+
+int nulpa_labels(nulpa_graph *g, int32_t *out, int memkind) {
+    if (!g || !out) return fail(NULPA_EINVAL, "null argument");
+    CHECK(resolve_mem(out, memkind));
+    CU(cudaMemcpyAsync(out, g->labels, g->n_global * sizeof(int32_t),
+                       memkind == NULPA_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    return NULPA_OK;
+}
+
+int nulpa_flags(nulpa_graph *g, uint8_t *out, int memkind) {
+    if (!g || !out) return fail(NULPA_EINVAL, "null argument");
+    CHECK(resolve_mem(out, memkind));
+    CU(cudaMemcpyAsync(out, g->flags, g->n_global,
+                       memkind == NULPA_MEM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    return NULPA_OK;
+}
+
+int nulpa_set_labels(nulpa_graph *g, const int32_t *in, const uint8_t *flags, int memkind) {
+    if (!g || !in) return fail(NULPA_EINVAL, "null argument");
+    CHECK(resolve_mem(in, memkind));
+    const cudaMemcpyKind k = memkind == NULPA_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+    CU(cudaMemcpyAsync(g->labels, in, g->n_global * sizeof(int32_t), k, g->stream));
+    if (flags)
+        CU(cudaMemcpyAsync(g->flags, flags, g->n_global, k, g->stream));
+    else
+        CU(cudaMemsetAsync(g->flags, 1, g->n_global, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    return NULPA_OK;
+}
+
+int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, double *sigma_intra, double *two_m,
+                             double *Sigma_device) {
+    if (!g || !sigma_intra || !two_m || !Sigma_device) return fail(NULPA_EINVAL, "null argument");
+    if (!g->macc) CHECK(dalloc(&g->macc, 4));
+    const int32_t *lab = labels_device ? labels_device : g->labels;
+    CU(cudaMemsetAsync(g->macc, 0, 4 * sizeof(double), g->stream));
+    const int grid = grid_for(g->n_rows, 8, num_sms() * 8);
+    if (g->weights)
+        k_mod_rows<true><<<grid, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, Sigma_device, g->macc);
+    else
+        k_mod_rows<false><<<grid, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, Sigma_device, g->macc);
+    CU(cudaGetLastError());
+    double h[4];
+    CU(cudaMemcpyAsync(h, g->macc, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    *sigma_intra += h[0];
+    *two_m += h[1];
+    return NULPA_OK;
+}
+
+int nulpa_modularity_finish(nulpa_graph *g, const double *Sigma_device, double sigma_intra, double two_m, double *q) {
+    if (!g || !Sigma_device || !q) return fail(NULPA_EINVAL, "null argument");
+    if (!g->macc) CHECK(dalloc(&g->macc, 4));
+    CU(cudaMemsetAsync(g->macc, 0, 4 * sizeof(double), g->stream));
+    k_mod_finish<<<grid_for(g->n_global, 256, num_sms() * 8), 256, 0, g->stream>>>(const_cast<double *>(Sigma_device), g->n_global, g->macc, 0);
+    CU(cudaGetLastError());
+    double h[4];
+    CU(cudaMemcpyAsync(h, g->macc, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    *q = two_m > 0 ? sigma_intra / two_m - h[2] / (two_m * two_m) : 0.0;
+    return NULPA_OK;
+}
+
+int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double *q) {
+    if (!g || !q) return fail(NULPA_EINVAL, "null argument");
+    if (g->n_rows != g->n_global) return fail(NULPA_ESTATE, "nulpa_modularity needs a whole graph; use the _partial/_finish pair for shards");
+    const int32_t *lab = g->labels;
+    int32_t *tmp = nullptr;
+    if (labels) {
+        CHECK(resolve_mem(labels, memkind));
+        if (memkind == NULPA_MEM_HOST) {
+            CHECK(dalloc(&tmp, (size_t)g->n_global));
+            CU(cudaMemcpyAsync(tmp, labels, g->n_global * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
+            lab = tmp;
+        } else {
+            lab = labels;
+        }
+    }
+    if (!g->Sigma) CHECK(dalloc(&g->Sigma, (size_t)g->n_global));
+    if (!g->macc) CHECK(dalloc(&g->macc, 4));
+    CU(cudaMemsetAsync(g->Sigma, 0, g->n_global * sizeof(double), g->stream));
+    double sigma = 0, two_m = 0;
+    int r = nulpa_modularity_partial(g, lab, &sigma, &two_m, g->Sigma);
+    if (r == NULPA_OK) r = nulpa_modularity_finish(g, g->Sigma, sigma, two_m, q);
+    cudaFree(tmp);
+    return r;
+}
+
+int nulpa_get_stats(nulpa_graph *g, nulpa_stats *out) {
+    if (!g || !out) return fail(NULPA_EINVAL, "null argument");
+    *out = g->stats;
+    return NULPA_OK;
+}
+
+int nulpa_state_pointers(nulpa_graph *g, int32_t **labels_device, uint8_t **flags_device) {
+    if (!g) return fail(NULPA_EINVAL, "null handle");
+    if (labels_device) *labels_device = g->labels;
+    if (flags_device) *flags_device = g->flags;
+    return NULPA_OK;
+}
+
+int nulpa_destroy(nulpa_graph *g) {
+    if (!g) return NULPA_OK;
+    if (g->stream) cudaStreamSynchronize(g->stream);
+    free_bins(g);
+    if (g->own_csr) {
+        cudaFree(g->offsets);
+        cudaFree(g->indices);
+        cudaFree(g->weights);
+    }
+    cudaFree(g->own_labels);
+    cudaFree(g->own_flags);
+    cudaFree(g->labels_prev);
+    cudaFree(g->flags_prev);
+    cudaFree(g->ctr);
+    if (g->ctr_host) cudaFreeHost(g->ctr_host);
+    cudaFree(g->Sigma);
+    cudaFree(g->macc);
+    if (g->events) {
+        for (auto &e : g->ev) cudaEventDestroy(e);
+        cudaEventDestroy(g->ev_run[0]);
+        cudaEventDestroy(g->ev_run[1]);
+    }
+    delete g;
+    return NULPA_OK;
+}
+
+}  // extern "C"

@@ -312,9 +312,11 @@ def kmer(n: int = 1_000_000, branch: float = 0.05, *, seed: int = 0, device="cpu
     return from_edges(torch.cat([a, xa]), torch.cat([b, xb]), n, weighted=weighted, seed=seed, name="kmer")
 
 
-def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.85, gamma: float = 3.6,
+def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.95, gamma: float = 3.6,
         host_alpha: float = 1.4, host_min: int = 16, host_max: int = 400_000, max_out: int = 20_000, *,
-        seed: int = 0, device="cpu", weighted: bool = False, chunk: int = 1 << 28) -> Graph:
+        locality: str = "loguniform", global_target: str = "page", seed: int = 0, device="cpu",
+        weighted: bool = False,
+        chunk: int = 1 << 28) -> Graph:
     """Web-graph-like power-law graph (BASELINE.json configs[4]: ~40M vertices /
     2.2B edges, it-2004-shaped).
 
@@ -322,7 +324,9 @@ def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.85, gamma
     a contiguous ID range (host sizes ~ Pareto(host_alpha) in
     [host_min, host_max]); out-degrees log-normal with mean `avg_out`; each
     link stays inside its host with probability p_local (uniform target),
-    otherwise it points to a globally popular page: rank floor(n * U^gamma)
+    uniform over the host (locality="uniform") or at a log-uniform ID distance
+    (locality="loguniform", the default: URL-ordered crawls link mostly to
+    nearby pages), otherwise it points to a globally popular page: rank floor(n * U^gamma)
     through a seeded permutation, which gives power-law in-degrees
     (rank^(1/gamma - 1)) and hubs with ~10^6 neighbours at full size."""
     g = _gen(seed, device)
@@ -342,6 +346,7 @@ def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.85, gamma
     z = torch.randn(n, generator=g, device=device)
     deg = torch.clamp(torch.exp(mu_ln + sigma * z).round().to(torch.int64), 1, max_out)
     perm = torch.randperm(n, generator=g, device=device)
+    hperm = torch.randperm(nh, generator=g, device=device)
     total = int(deg.sum())
     srcs, dsts = [], []
     cdeg = torch.cumsum(deg, 0)
@@ -358,9 +363,24 @@ def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.85, gamma
         h = host_of[src]
         loc = torch.rand(cnt, generator=g, device=device) < p_local
         r = torch.rand(cnt, generator=g, device=device, dtype=torch.float64)
-        dl = hstart[h] + (r * hs[h]).to(torch.int64)
+        if locality == "uniform":
+            dl = hstart[h] + (r * hs[h]).to(torch.int64)
+        else:
+            # URL-order locality: distance to the target page log-uniform in
+            # [1, host size], either direction, wrapped inside the host
+            hsz = hs[h]
+            dist = torch.exp(r * torch.log(hsz.to(torch.float64))).to(torch.int64)
+            sign = torch.rand(cnt, generator=g, device=device) < 0.5
+            dist = torch.where(sign, dist, -dist)
+            dl = hstart[h] + torch.remainder(src - hstart[h] + dist, hsz)
         r2 = torch.rand(cnt, generator=g, device=device, dtype=torch.float64)
-        dg = perm[torch.clamp((n * r2.pow(gamma)).to(torch.int64), max=n - 1)]
+        if global_target == "page":
+            dg = perm[torch.clamp((n * r2.pow(gamma)).to(torch.int64), max=n - 1)]
+        else:
+            # links into another host land on its home page (first ID of the
+            # host: the root URL sorts first); hosts chosen by popularity
+            hp = hperm[torch.clamp((nh * r2.pow(gamma)).to(torch.int64), max=nh - 1)]
+            dg = hstart[hp]
         dst = torch.where(loc, dl, dg)
         srcs.append(src)
         dsts.append(dst)
