@@ -23,7 +23,6 @@
 #include "nulpa.h"
 
 #include <cuda_runtime.h>
-#include <cub/device/device_scan.cuh>
 
 #include <algorithm>
 #include <cstdarg>
@@ -41,7 +40,8 @@ constexpr int kCtr = 24;                 // counters per iteration
 // counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
 
 constexpr int kWarpThreads = 256;        // k_warp: 8 warps per CTA
-constexpr int kWarpCap = 256;            // slots per warp table (degree <= 255 -> p1 <= 255)
+constexpr int kWarpCap = 256;            // degree bound of the warp bin (degree <= 255)
+constexpr int kWarpTab = 256;            // slots of a k_warp table (P1 = 255)
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
 constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
 constexpr int kGiantChunk = 4096;        // edges per giant chunk
@@ -128,15 +128,14 @@ struct Hash {
 // rule 1 uses (k mod p1) * Q + (k div p1) with Q = floor((2^31-1)/p1) + 1,
 // a bijection onto [0, p1*Q) < 2^32; (k div p1) is the exact division
 // (k - k mod p1) * p1^-1 mod 2^32 (p1 = 2^a - 1 is odd).
+template <int RULE>
 struct TieOrder {
-    int rule;
     uint32_t p1, Q, inv;
     uint64_t m1;
-    __device__ __forceinline__ void init(int r, const Hash &h) {
-        rule = r;
-        p1 = h.p1;
-        m1 = h.m1;
-        if (r) {
+    __device__ __forceinline__ void init(const Hash &h) {
+        if (RULE) {
+            p1 = h.p1;
+            m1 = h.m1;
             Q = p1 ? 0x7FFFFFFFu / p1 + 1 : 1;
             uint32_t x = p1;                       // Newton: x <- x (2 - p1 x)
 #pragma unroll
@@ -145,13 +144,13 @@ struct TieOrder {
         }
     }
     __device__ __forceinline__ uint32_t rank(int32_t k) const {
-        if (!rule) return (uint32_t)k;
-        uint32_t home = fastmod((uint32_t)k, m1, p1);
+        if (!RULE) return (uint32_t)k;
+        const uint32_t home = fastmod((uint32_t)k, m1, p1);
         return home * Q + ((uint32_t)k - home) * inv;
     }
     __device__ __forceinline__ int32_t unrank(uint32_t t) const {
-        if (!rule) return (int32_t)t;
-        uint32_t home = t / Q;
+        if (!RULE) return (int32_t)t;
+        const uint32_t home = t / Q;
         return (int32_t)((t - home * Q) * p1 + home);
     }
 };
@@ -253,6 +252,55 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
     return x;
 }
 
+// Warp-private TAGGED table (k_warp): slot s holds tk[s] = (tag << 32) | key
+// and tv[s]; a slot whose tag is not the current vertex's tag is empty (phi),
+// so a table never needs hashtableClear -- every vertex gets a fresh tag.
+// B200 design change: the table lives in shared memory and is reused by all
+// vertices the warp processes, so its capacity P1 = 511 (p2 = 1023) is set by
+// the shared-memory budget instead of nextPow2(D)-1 (PAPER.md:208 sizes the
+// per-vertex GLOBAL tables that way; the giant bin keeps that sizing).  At
+// degree < 256 the load factor stays below 1/2, so probes rarely collide.
+// tt_add is Algorithm 2's accumulate (hybrid quadratic-double probing from
+// slot k mod p1, R5 linear continuation) for a leader adding its group's
+// weight x; it returns the label's new total.  Keys within one batch are
+// distinct (one leader per label), batches are ordered by __syncwarp, so the
+// value update is a plain read-modify-write; only the slot claim is atomic
+// (64-bit shared-memory CAS).
+template <uint32_t P1>
+__device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, int32_t k, float x) {
+    constexpr uint32_t p1 = P1, p2 = 2 * P1 + 1;
+    const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
+    uint32_t i = (uint32_t)k % p1;
+    uint32_t di = 1;
+    uint32_t km = 0xFFFFFFFFu;                             // k mod p2, computed on the first collision
+    for (int t = 0;; ++t) {
+        const uint64_t cur = *((volatile uint64_t *)&tk[i]);
+        if (cur == want) {
+            const float V = __fadd_rn(tv[i], x);
+            tv[i] = V;
+            return V;
+        }
+        if ((uint32_t)(cur >> 32) != tag) {                 // empty slot: claim it
+            const unsigned long long old =
+                atomicCAS((unsigned long long *)&tk[i], (unsigned long long)cur, (unsigned long long)want);
+            if (old == cur) {
+                tv[i] = x;
+                return x;
+            }
+        }
+        if (t < kMaxRetries) {
+            if (km == 0xFFFFFFFFu) km = ((uint32_t)k % p2) % p1;
+            i += di;
+            if (i >= p1) i -= p1;
+            di = 2 * di + km;
+            if (di >= p1) di -= p1;
+            if (di >= p1) di -= p1;
+        } else {
+            i = i + 1 == p1 ? 0 : i + 1;                   // R5
+        }
+    }
+}
+
 // One 32-edge batch of a warp against the warp's PRIVATE table: lanes
 // holding the same label (match_any) are folded onto their lowest lane (the
 // leader), which claims the label's slot (Algorithm 2 probing, atomicCAS on
@@ -303,10 +351,12 @@ __device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float 
 // (weight, tie rank) packed so that an unsigned max gives the largest weight
 // and, among equal weights, the label first in tie order (R6; R12: weights
 // >= 0 so IEEE bit patterns order like the values).  0 = no candidate.
-__device__ __forceinline__ uint64_t pack_cand(float w, int32_t k, const TieOrder &to) {
+template <int RULE>
+__device__ __forceinline__ uint64_t pack_cand(float w, int32_t k, const TieOrder<RULE> &to) {
     return ((uint64_t)__float_as_uint(w) << 32) | (uint64_t)(0xFFFFFFFFu - to.rank(k));
 }
-__device__ __forceinline__ int32_t cand_label(uint64_t c, const TieOrder &to) {
+template <int RULE>
+__device__ __forceinline__ int32_t cand_label(uint64_t c, const TieOrder<RULE> &to) {
     return to.unrank(0xFFFFFFFFu - (uint32_t)(c & 0xFFFFFFFFu));
 }
 __device__ __forceinline__ uint64_t warp_max_u64(uint64_t x) {
@@ -333,7 +383,6 @@ struct SweepArgs {
     uint8_t *flag_out;
     int64_t row_begin;
     int pickless;
-    int tie_rule;
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 
@@ -372,7 +421,7 @@ __device__ __forceinline__ void block_count(unsigned long long *ctr, unsigned lo
 // lab[m] == lab[k], taken in CSR order (bit-identical to a sequential
 // float32 hashtable accumulation).
 // ---------------------------------------------------------------------------
-template <bool SYNC, bool W, int MAXD>
+template <bool SYNC, bool W, int TIE, int MAXD>
 __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const int32_t *__restrict__ list,
                                                            int64_t n) {
     __shared__ unsigned long long bctr[4];
@@ -405,8 +454,8 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
             }
             Hash h;
             h.init(deg);
-            TieOrder to;
-            to.init(a.tie_rule, h);
+            TieOrder<TIE> to;
+            to.init(h);
             uint64_t best = 0;
 #pragma unroll
             for (int k = 0; k < MAXD; ++k) {
@@ -437,21 +486,33 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
 // warp-per-vertex kernel: one 32-lane warp per vertex, the vertex's table
 // (p1 <= 255 slots) in shared memory, persistent grid-stride over the bin.
 // ---------------------------------------------------------------------------
-template <bool SYNC, bool W>
-__global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_t *__restrict__ list,
-                                                       int64_t n) {
-    __shared__ int32_t sk[kWarpThreads / 32][kWarpCap];
-    __shared__ float sv[kWarpThreads / 32][kWarpCap];
+__device__ __forceinline__ void cp_async4(void *smem, const void *gmem) {
+    const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(sa), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+// Per-warp shared memory of k_warp: the tagged table.
+struct WarpSmem {
+    uint64_t tk[kWarpTab];
+    float tv[kWarpTab];
+};
+
+template <bool SYNC, bool W, int TIE>
+__global__ void __launch_bounds__(kWarpThreads, 6) k_warp(SweepArgs a, const int32_t *__restrict__ list,
+                                                          int64_t n) {
+    extern __shared__ __align__(16) unsigned char wsm[];
     __shared__ unsigned long long bctr[4];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    int32_t *Hk = sk[wid];
-    float *Hv = sv[wid];
-    for (int s = lane; s < kWarpCap; s += 32) {
-        Hk[s] = kEmpty;
-        Hv[s] = 0.0f;
-    }
+    WarpSmem &S = reinterpret_cast<WarpSmem *>(wsm)[wid];
+    uint64_t *tk = S.tk;
+    float *tv = S.tv;
+    for (int q = lane; q < kWarpTab; q += 32) tk[q] = 0;   // tag 0: empty for every vertex
     if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
     __syncthreads();
+    uint32_t tag = 0;
     unsigned long long c_act = 0, c_edges = 0, c_ch = 0, c_che = 0;   // lane 0's tallies
     const int64_t nw = (int64_t)gridDim.x * (kWarpThreads / 32);
     const int64_t nchunks = (n + 31) / 32;
@@ -485,9 +546,10 @@ __global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_
             const int64_t vk = rk + a.row_begin;
             Hash h;
             h.init(dk);
-            // the first 64 entries of the row stay in registers (degree < 64
-            // covers most vertices); indices/weights first, then all the
-            // neighbour labels: two dependent round trips per vertex
+            TieOrder<TIE> to;
+            to.init(h);
+            // the first 64 entries of the row stay in registers; indices and
+            // weights first, then all the neighbour labels
             const bool v0 = (uint32_t)lane < dk, v1 = (uint32_t)(lane + 32) < dk;
             const int32_t j0 = v0 ? a.indices[ok + lane] : -1;
             const int32_t j1 = v1 ? a.indices[ok + 32 + lane] : -1;
@@ -498,36 +560,64 @@ __global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_
             }
             const int32_t k0 = (j0 >= 0 && j0 != (int32_t)vk) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
             const int32_t k1 = (j1 >= 0 && j1 != (int32_t)vk) ? a.lab_in[j1] : kEmpty;
-            warp_batch_accumulate<W>(Hk, Hv, h, k0, w0);
-            if (dk > 32) warp_batch_accumulate<W>(Hk, Hv, h, k1, w1);
-            for (uint32_t b = 64; b < dk; b += 64) {
-                const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
-                const int32_t i0 = u0 ? a.indices[ok + b + lane] : -1;
-                const int32_t i1 = u1 ? a.indices[ok + b + 32 + lane] : -1;
-                float x0 = 0.0f, x1 = 0.0f;
+            // per-lane running best (weight bits + 1, label) over the label
+            // totals this lane produced as a group leader; the maximum over
+            // all lanes is hashtableMaxKey (totals only grow, so partial
+            // totals never exceed the final maximum)
+            uint32_t bw = 0;
+            int32_t bk = 0;
+            auto offer = [&](float V, int32_t key) {
+                const uint32_t vb = __float_as_uint(V) + 1;
+                if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
+                    bw = vb;
+                    bk = key;
+                }
+            };
+            auto fold = [&](int32_t key, float w, unsigned &grp) -> float {
+                grp = __match_any_sync(0xFFFFFFFFu, key);
                 if (W) {
-                    if (u0) x0 = a.weights[ok + b + lane];
-                    if (u1) x1 = a.weights[ok + b + 32 + lane];
+                    const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+                    return maxn > 1 ? group_sum(grp, w, maxn) : w;
                 }
-                const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
-                const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
-                warp_batch_accumulate<W>(Hk, Hv, h, q0, x0);
-                if (b + 32 < dk) warp_batch_accumulate<W>(Hk, Hv, h, q1, x1);
-            }
-            TieOrder to;
-            to.init(a.tie_rule, h);
-            uint64_t best = 0;
-            for (uint32_t s = lane; s < h.p1; s += 32) {    // hashtableMaxKey + clear
-                const int32_t key = Hk[s];
-                if (key != kEmpty) {
-                    const uint64_t cd = pack_cand(Hv[s], key, to);
-                    best = cd > best ? cd : best;
-                    Hk[s] = kEmpty;
-                    Hv[s] = 0.0f;
+                return (float)__popc(grp);
+            };
+            if (dk <= 32) {
+                // one batch: the match_any groups ARE the label totals -- no table
+                unsigned grp;
+                const float x = fold(k0, w0, grp);
+                if (k0 != kEmpty && lane == __ffs(grp) - 1) offer(x, k0);
+            } else {
+                ++tag;
+                auto batch = [&](int32_t key, float w) {
+                    unsigned grp;
+                    const float x = fold(key, w, grp);
+                    if (key != kEmpty && lane == __ffs(grp) - 1) offer(tt_add<kWarpTab - 1>(tk, tv, tag, key, x), key);
+                    __syncwarp();
+                };
+                batch(k0, w0);
+                batch(k1, w1);
+                for (uint32_t b = 64; b < dk; b += 64) {
+                    const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
+                    const int32_t i0 = u0 ? a.indices[ok + b + lane] : -1;
+                    const int32_t i1 = u1 ? a.indices[ok + b + 32 + lane] : -1;
+                    float x0 = 0.0f, x1 = 0.0f;
+                    if (W) {
+                        if (u0) x0 = a.weights[ok + b + lane];
+                        if (u1) x1 = a.weights[ok + b + 32 + lane];
+                    }
+                    const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
+                    const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
+                    batch(q0, x0);
+                    if (b + 32 < dk) batch(q1, x1);
                 }
             }
-            best = warp_max_u64(best);
-            const int32_t cs = best ? cand_label(best, to) : kEmpty;
+            // hashtableMaxKey: max weight, then first label in tie order
+            const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
+            int32_t cs = kEmpty;
+            if (W1) {
+                const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
+                cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
+            }
             const bool changed = accept_move(cs, cik, a.pickless);
             if (changed) {
                 if (lane == 0) a.lab_out[vk] = cs;
@@ -535,7 +625,6 @@ __global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_
                 if (j1 >= 0) a.flag_out[j1] = 1;
                 for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[a.indices[ok + b]] = 1;
             }
-            __syncwarp();
             c_act += 1;
             c_edges += dk;
             c_ch += changed;
@@ -561,238 +650,10 @@ __global__ void __launch_bounds__(kWarpThreads) k_warp(SweepArgs a, const int32_
 }
 
 // ---------------------------------------------------------------------------
-// tile kernel (the warp bin, switch_degree <= degree < block_degree): the
-// bin is cut into tiles of consecutive bin entries holding ~kTileE first
-// edges (<= kTileV vertices).  A CTA (8 warps) processes a tile in phases:
-//   1. metadata of all tile vertices (row, flag, offsets, own label) in one
-//      round trip, one thread per vertex; an exclusive scan places the
-//      active rows back to back in shared memory;
-//   2. the active rows' indices / weights are staged into shared memory with
-//      cp.async (LDGSTS, no register round trip; many copies in flight);
-//   3. the neighbour labels are gathered, ~9 independent loads per thread;
-//   4. each warp runs Algorithm 1's per-vertex body for its vertices from
-//      shared memory: fold the row into the warp-private table
-//      (warp_batch_accumulate), hashtableMaxKey, move rule, mark neighbours.
-// Global-memory latency is paid a few times per tile instead of per vertex.
-// ---------------------------------------------------------------------------
-constexpr int kTileThreads = 256;
-constexpr int kTileE = 2048;                 // first-edge budget of a tile
-constexpr int kTileV = 256;                  // vertices per tile (one per thread)
-constexpr int kTileSlots = kTileE + kWarpCap; // + the last vertex's degree (< 256)
-
-template <bool W>
-struct TileSmem {
-    int32_t hk[kTileThreads / 32][kWarpCap];
-    float hv[kTileThreads / 32][kWarpCap];
-    int32_t idx[kTileSlots];
-    int32_t lab[kTileSlots];
-    float w[W ? kTileSlots : 1];
-    int64_t o[kTileV];
-    int32_t r[kTileV];
-    int32_t deg[kTileV];
-    int32_t ci[kTileV];
-    int32_t pfx[kTileV + 1];
-    int32_t act[kTileV];
-    int32_t wsum[kTileThreads / 32];
-    int32_t nact;
-    unsigned long long bctr[4];
-};
-
-__device__ __forceinline__ void cp_async4(void *smem, const void *gmem) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
-
-template <bool SYNC, bool W>
-__global__ void __launch_bounds__(kTileThreads, 4) k_tile(SweepArgs a, const int32_t *__restrict__ list,
-                                                           const int32_t *__restrict__ tile_start, int64_t ntiles) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    TileSmem<W> &S = *reinterpret_cast<TileSmem<W> *>(smem_raw);
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    int32_t *Hk = S.hk[wid];
-    float *Hv = S.hv[wid];
-    for (int q = lane; q < kWarpCap; q += 32) {
-        Hk[q] = kEmpty;
-        Hv[q] = 0.0f;
-    }
-    if (tid < 4) S.bctr[tid] = 0;
-    unsigned long long c_act = 0, c_edges = 0, c_ch = 0, c_che = 0;   // lane 0's tallies
-    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const int32_t k0 = tile_start[tile];
-        const int nv = tile_start[tile + 1] - k0;
-        // -- phase 1: metadata, one thread per vertex ------------------------
-        int32_t d = 0;
-        if (tid < nv) {
-            const int32_t r = list[k0 + tid];
-            const int64_t v = r + a.row_begin;
-            S.r[tid] = r;
-            if (a.flag_in[v]) {
-                const int64_t o = a.offsets[r];
-                d = (int32_t)(a.offsets[r + 1] - o);
-                S.o[tid] = o;
-                S.ci[tid] = a.lab_in[v];
-                if (!SYNC) a.flag_in[v] = 0;                // mark i as processed
-            }
-            S.deg[tid] = d;
-        }
-        // exclusive scan of active degrees + compaction of active slots
-        int32_t x = d;
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const int32_t y = __shfl_up_sync(0xFFFFFFFFu, x, off);
-            if (lane >= off) x += y;
-        }
-        const unsigned am = __ballot_sync(0xFFFFFFFFu, d > 0);
-        if (lane == 31) S.wsum[wid] = x;
-        __shared__ int32_t wact[kTileThreads / 32];
-        if (lane == 0) wact[wid] = __popc(am);
-        __syncthreads();
-        int32_t base = 0, abase = 0;
-        for (int q = 0; q < wid; ++q) {
-            base += S.wsum[q];
-            abase += wact[q];
-        }
-        S.pfx[tid] = base + x - d;
-        if (d > 0) S.act[abase + __popc(am & ((1u << lane) - 1))] = tid;
-        if (tid == kTileThreads - 1) {
-            S.pfx[kTileV] = base + x;
-            S.nact = abase + __popc(am);
-        }
-        __syncthreads();
-        const int nact = S.nact;
-        const int32_t total = S.pfx[kTileV];
-        // -- phase 2: stage the active rows with cp.async --------------------
-        for (int q = wid; q < nact; q += kTileThreads / 32) {
-            const int kk = S.act[q];
-            const int64_t o = S.o[kk];
-            const int32_t dk = S.deg[kk], p0 = S.pfx[kk];
-            for (int e = lane; e < dk; e += 32) {
-                cp_async4(&S.idx[p0 + e], a.indices + o + e);
-                if (W) cp_async4(&S.w[p0 + e], a.weights + o + e);
-            }
-        }
-        cp_async_wait_all();
-        __syncthreads();
-        // -- phase 3: gather neighbour labels --------------------------------
-        for (int p = tid; p < total; p += 4 * kTileThreads) {
-            int32_t j[4], l[4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u) j[u] = p + u * kTileThreads < total ? S.idx[p + u * kTileThreads] : -1;
-#pragma unroll
-            for (int u = 0; u < 4; ++u) l[u] = j[u] >= 0 ? a.lab_in[j[u]] : kEmpty;
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-                if (j[u] >= 0) S.lab[p + u * kTileThreads] = l[u];
-        }
-        __syncthreads();
-        // -- phase 4: per-vertex body, one warp per vertex -------------------
-        for (int q = wid; q < nact; q += kTileThreads / 32) {
-            const int kk = S.act[q];
-            const int64_t vk = S.r[kk] + a.row_begin;
-            const uint32_t dk = (uint32_t)S.deg[kk];
-            const int32_t p0 = S.pfx[kk];
-            Hash h;
-            h.init(dk);
-            for (uint32_t b = 0; b < dk; b += 32) {
-                int32_t key = kEmpty;
-                float w = 0.0f;
-                if (b + lane < dk) {
-                    const int32_t p = p0 + (int32_t)(b + lane);
-                    if (S.idx[p] != (int32_t)vk) {           // "if j = i continue"
-                        key = S.lab[p];
-                        if (W) w = S.w[p];
-                    }
-                }
-                warp_batch_accumulate<W>(Hk, Hv, h, key, w);
-            }
-            TieOrder to;
-            to.init(a.tie_rule, h);
-            uint64_t best = 0;
-            for (uint32_t sl = lane; sl < h.p1; sl += 32) { // hashtableMaxKey + clear
-                const int32_t key = Hk[sl];
-                if (key != kEmpty) {
-                    const uint64_t cd = pack_cand(Hv[sl], key, to);
-                    best = cd > best ? cd : best;
-                    Hk[sl] = kEmpty;
-                    Hv[sl] = 0.0f;
-                }
-            }
-            best = warp_max_u64(best);
-            const int32_t cs = best ? cand_label(best, to) : kEmpty;
-            const bool changed = accept_move(cs, S.ci[kk], a.pickless);
-            if (changed) {
-                if (lane == 0) a.lab_out[vk] = cs;
-                for (uint32_t b = lane; b < dk; b += 32) a.flag_out[S.idx[p0 + b]] = 1;   // mark neighbours
-            }
-            __syncwarp();
-            c_act += 1;
-            c_edges += dk;
-            c_ch += changed;
-            c_che += changed ? dk : 0;
-        }
-        __syncthreads();
-    }
-    if (lane == 0 && c_act) {
-        atomicAdd(&S.bctr[0], c_act);
-        atomicAdd(&S.bctr[1], c_edges);
-        atomicAdd(&S.bctr[2], c_ch);
-        atomicAdd(&S.bctr[3], c_che);
-    }
-    __syncthreads();
-    if (tid == 0 && S.bctr[0]) {
-        atomicAdd(&a.ctr[1 + 1], S.bctr[0]);
-        atomicAdd(&a.ctr[5 + 1], S.bctr[1]);
-        if (S.bctr[2]) {
-            atomicAdd(&a.ctr[0], S.bctr[2]);
-            atomicAdd(&a.ctr[9 + 1], S.bctr[2]);
-            atomicAdd(&a.ctr[13 + 1], S.bctr[3]);
-        }
-    }
-}
-
-// tile construction: degree of every bin entry; tiles of ~kTileE first edges
-__global__ void k_bin_entry_degrees(const int64_t *offsets, const int32_t *list, int64_t n, int64_t *deg) {
-    const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (k < n) deg[k] = offsets[list[k] + 1] - offsets[list[k]];
-    if (k == n) deg[k] = 0;
-}
-// coarse tile t starts at the first entry whose first edge is >= t*kTileE;
-// count of sub-tiles of <= kTileV entries per coarse tile
-__global__ void k_tile_coarse(const int64_t *pfx, int64_t n, int64_t ncoarse, int64_t *ks, int64_t *nsub) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t > ncoarse) return;
-    int64_t lo = 0, hi = n;                      // first k in [0, n] with pfx[k] >= t*E
-    const int64_t target = t * kTileE;
-    if (t == ncoarse) {
-        lo = n;
-    } else {
-        while (lo < hi) {
-            const int64_t mid = (lo + hi) >> 1;
-            if (pfx[mid] < target) lo = mid + 1; else hi = mid;
-        }
-    }
-    ks[t] = lo;
-}
-__global__ void k_tile_count(const int64_t *ks, int64_t ncoarse, int64_t *nsub) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t < ncoarse) nsub[t] = (ks[t + 1] - ks[t] + kTileV - 1) / kTileV;
-    if (t == ncoarse) nsub[t] = 0;
-}
-__global__ void k_tile_emit(const int64_t *ks, const int64_t *nsub_pfx, int64_t ncoarse, int64_t n, int32_t *tile_start) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t < ncoarse) {
-        const int64_t b = nsub_pfx[t], e = nsub_pfx[t + 1];
-        for (int64_t q = b; q < e; ++q) tile_start[q] = (int32_t)(ks[t] + (q - b) * kTileV);
-    }
-    if (t == ncoarse) tile_start[nsub_pfx[ncoarse]] = (int32_t)n;
-}
-
-// ---------------------------------------------------------------------------
 // block-per-vertex kernel: one CTA per vertex, table (p1 <= 4095) in dynamic
 // shared memory, persistent grid-stride over the bin.  PAPER.md:243.
 // ---------------------------------------------------------------------------
-template <bool SYNC, bool W>
+template <bool SYNC, bool W, int TIE>
 __global__ void __launch_bounds__(kBlockThreads) k_block(SweepArgs a, const int32_t *__restrict__ list,
                                                          int64_t n) {
     extern __shared__ int32_t dyn[];
@@ -835,8 +696,8 @@ __global__ void __launch_bounds__(kBlockThreads) k_block(SweepArgs a, const int3
                 warp_batch_accumulate_atomic<W>(Hk, Hv, h, key, w);
             }
             __syncthreads();
-            TieOrder to;
-            to.init(a.tie_rule, h);
+            TieOrder<TIE> to;
+            to.init(h);
             uint64_t best = 0;
             for (uint32_t s = threadIdx.x; s < h.p1; s += kBlockThreads) {
                 int32_t k = Hk[s];
@@ -962,7 +823,7 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
     if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
 }
 
-template <bool SYNC>
+template <bool SYNC, int TIE>
 __global__ void __launch_bounds__(kBlockThreads) k_giant_finalize(SweepArgs a, GiantArgs g) {
     const int64_t gi = blockIdx.x;
     if (!g.active[gi]) return;
@@ -975,8 +836,8 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_finalize(SweepArgs a, G
     const int32_t r = g.verts[gi];
     Hash h;
     h.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
-    TieOrder to;
-    to.init(a.tie_rule, h);
+    TieOrder<TIE> to;
+    to.init(h);
     uint64_t best = 0;
     for (int32_t q = threadIdx.x; q < cnt; q += kBlockThreads) {
         int32_t s = occ[q];
@@ -1256,10 +1117,6 @@ struct nulpa_graph {
     int32_t *gkeys = nullptr, *occ = nullptr, *occ_n = nullptr;
     float *gvals = nullptr;
     uint8_t *gactive = nullptr, *gchanged = nullptr;
-    // tiles of the warp bin
-    int64_t n_tiles = 0;
-    int32_t *tile_start = nullptr;
-    int warp_kernel = 0;                     // 0: k_tile, 1: k_warp (env NULPA_WARP_KERNEL)
     // counters
     unsigned long long *ctr = nullptr;       // device [kMaxIter+1][kCtr]
     unsigned long long *ctr_host = nullptr;  // pinned
@@ -1303,9 +1160,6 @@ void free_bins(nulpa_graph *g) {
     cudaFree(g->occ_n);
     cudaFree(g->gactive);
     cudaFree(g->gchanged);
-    cudaFree(g->tile_start);
-    g->tile_start = nullptr;
-    g->n_tiles = 0;
     g->chunk_g = nullptr;
     g->chunk_e0 = g->chunk_e1 = g->table_off = nullptr;
     g->gkeys = g->occ = g->occ_n = nullptr;
@@ -1363,53 +1217,6 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
     if (nb > 0) {
         k_bin_scatter<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, L);
         CU(cudaGetLastError());
-    }
-    // tiles of the warp bin (k_tile)
-    if (g->bin_n[1] > 0) {
-        const int64_t n1 = g->bin_n[1];
-        int64_t *deg1 = nullptr, *pfx1 = nullptr;
-        CHECK(dalloc(&deg1, (size_t)n1 + 1));
-        CHECK(dalloc(&pfx1, (size_t)n1 + 1));
-        k_bin_entry_degrees<<<grid_for(n1 + 1, 256), 256, 0, g->stream>>>(g->offsets, g->bin_list[1], n1, deg1);
-        CU(cudaGetLastError());
-        size_t tmp_bytes = 0;
-        CU(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, deg1, pfx1, n1 + 1, g->stream));
-        void *tmp = nullptr;
-        CU(cudaMalloc(&tmp, tmp_bytes));
-        CU(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, deg1, pfx1, n1 + 1, g->stream));
-        int64_t E1 = 0;
-        CU(cudaMemcpyAsync(&E1, pfx1 + n1, sizeof E1, cudaMemcpyDeviceToHost, g->stream));
-        CU(cudaStreamSynchronize(g->stream));
-        const int64_t ncoarse = (E1 + kTileE - 1) / kTileE;
-        int64_t *ks = nullptr, *nsub = nullptr, *nsub_pfx = nullptr;
-        CHECK(dalloc(&ks, (size_t)ncoarse + 1));
-        CHECK(dalloc(&nsub, (size_t)ncoarse + 1));
-        CHECK(dalloc(&nsub_pfx, (size_t)ncoarse + 1));
-        k_tile_coarse<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(pfx1, n1, ncoarse, ks, nsub);
-        k_tile_count<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(ks, ncoarse, nsub);
-        CU(cudaGetLastError());
-        size_t tmp2 = 0;
-        CU(cub::DeviceScan::ExclusiveSum(nullptr, tmp2, nsub, nsub_pfx, ncoarse + 1, g->stream));
-        if (tmp2 > tmp_bytes) {
-            cudaFree(tmp);
-            CU(cudaMalloc(&tmp, tmp2));
-            tmp_bytes = tmp2;
-        }
-        CU(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, nsub, nsub_pfx, ncoarse + 1, g->stream));
-        int64_t nt = 0;
-        CU(cudaMemcpyAsync(&nt, nsub_pfx + ncoarse, sizeof nt, cudaMemcpyDeviceToHost, g->stream));
-        CU(cudaStreamSynchronize(g->stream));
-        g->n_tiles = nt;
-        CHECK(dalloc(&g->tile_start, (size_t)nt + 1));
-        k_tile_emit<<<grid_for(ncoarse + 1, 256), 256, 0, g->stream>>>(ks, nsub_pfx, ncoarse, n1, g->tile_start);
-        CU(cudaGetLastError());
-        CU(cudaStreamSynchronize(g->stream));
-        cudaFree(tmp);
-        cudaFree(deg1);
-        cudaFree(pfx1);
-        cudaFree(ks);
-        cudaFree(nsub);
-        cudaFree(nsub_pfx);
     }
     // giant chunks (host-side bookkeeping over the few giant vertices)
     const int64_t ng = g->bin_n[3];
@@ -1490,26 +1297,25 @@ int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
     return build_bins(g, p.switch_degree, p.block_degree, p.giant_degree);
 }
 
-template <bool SYNC, bool W>
+template <bool SYNC, bool W, int TIE>
 int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const int64_t n = g->bin_n[0];
     const int grid = grid_for(n, kThreadThreads);
     if (g->t1 <= 5)
-        k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, TIE, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else if (g->t1 <= 9)
-        k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, TIE, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else if (g->t1 <= 17)
-        k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, TIE, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else
-        k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, TIE, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     CU(cudaGetLastError());
     return NULPA_OK;
 }
 
-template <bool SYNC, bool W>
+template <bool SYNC, bool W, int TIE>
 int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
     SweepArgs a;
-    a.tie_rule = p.tie_rule;
     a.offsets = g->offsets;
     a.indices = g->indices;
     a.weights = g->weights;
@@ -1558,7 +1364,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             }
             k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, g->stream>>>(a, ga, ng);
             k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, g->stream>>>(a, ga);
-            k_giant_finalize<SYNC><<<(unsigned)ng, kBlockThreads, 0, g->stream>>>(a, ga);
+            k_giant_finalize<SYNC, TIE><<<(unsigned)ng, kBlockThreads, 0, g->stream>>>(a, ga);
             k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
             CU(cudaGetLastError());
             g->stats.launches[3] += 4;
@@ -1571,7 +1377,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(2, 0));
         if (n > 0) {
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W><<<grid_for(n, 1, sms * 4), kBlockThreads, smem, g->stream>>>(a, g->bin_list[2], n);
+            k_block<SYNC, W, TIE><<<grid_for(n, 1, sms * 4), kBlockThreads, smem, g->stream>>>(a, g->bin_list[2], n);
             CU(cudaGetLastError());
             g->stats.launches[2] += 1;
         }
@@ -1582,18 +1388,12 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[1];
         CHECK(rec(1, 0));
         if (n > 0) {
-            if (g->warp_kernel == 0) {
-                const size_t smem = sizeof(TileSmem<W>);
-                static bool attr_set = false;
-                if (!attr_set) {
-                    CU(cudaFuncSetAttribute(k_tile<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-                    attr_set = true;
-                }
-                k_tile<SYNC, W><<<grid_for(g->n_tiles, 1, sms * 4), kTileThreads, smem, g->stream>>>(
-                    a, g->bin_list[1], g->tile_start, g->n_tiles);
-            } else {
-                k_warp<SYNC, W><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * 8), kWarpThreads, 0, g->stream>>>(a, g->bin_list[1], n);
+            static bool attr_set = false;
+            if (!attr_set) {
+                CU(cudaFuncSetAttribute(k_warp<SYNC, W, TIE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(WarpSmem) * (kWarpThreads / 32))));
+                attr_set = true;
             }
+            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * 6), kWarpThreads, sizeof(WarpSmem) * (kWarpThreads / 32), g->stream>>>(a, g->bin_list[1], n);
             CU(cudaGetLastError());
             g->stats.launches[1] += 1;
         }
@@ -1604,7 +1404,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[0];
         CHECK(rec(0, 0));
         if (n > 0) {
-            CHECK((launch_thread_bin<SYNC, W>(g, a)));
+            CHECK((launch_thread_bin<SYNC, W, TIE>(g, a)));
             g->stats.launches[0] += 1;
         }
         CHECK(rec(0, 1));
@@ -1626,14 +1426,21 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
 
 int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
     const bool w = g->weights != nullptr;
-    if (p.mode == NULPA_SYNC) {
-        if (!g->labels_prev) {
-            CHECK(dalloc(&g->labels_prev, (size_t)g->n_global));
-            CHECK(dalloc(&g->flags_prev, (size_t)g->n_global));
-        }
-        return w ? sweep_impl<true, true>(g, pickless, p, ctr, timing, slot) : sweep_impl<true, false>(g, pickless, p, ctr, timing, slot);
+    if (p.mode == NULPA_SYNC && !g->labels_prev) {
+        CHECK(dalloc(&g->labels_prev, (size_t)g->n_global));
+        CHECK(dalloc(&g->flags_prev, (size_t)g->n_global));
     }
-    return w ? sweep_impl<false, true>(g, pickless, p, ctr, timing, slot) : sweep_impl<false, false>(g, pickless, p, ctr, timing, slot);
+    const int sel = (p.mode == NULPA_SYNC ? 4 : 0) + (w ? 2 : 0) + (p.tie_rule ? 1 : 0);
+    switch (sel) {
+    case 0: return sweep_impl<false, false, 0>(g, pickless, p, ctr, timing, slot);
+    case 1: return sweep_impl<false, false, 1>(g, pickless, p, ctr, timing, slot);
+    case 2: return sweep_impl<false, true, 0>(g, pickless, p, ctr, timing, slot);
+    case 3: return sweep_impl<false, true, 1>(g, pickless, p, ctr, timing, slot);
+    case 4: return sweep_impl<true, false, 0>(g, pickless, p, ctr, timing, slot);
+    case 5: return sweep_impl<true, false, 1>(g, pickless, p, ctr, timing, slot);
+    case 6: return sweep_impl<true, true, 0>(g, pickless, p, ctr, timing, slot);
+    default: return sweep_impl<true, true, 1>(g, pickless, p, ctr, timing, slot);
+    }
 }
 
 int reset_state(nulpa_graph *g) {
@@ -1705,7 +1512,6 @@ int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *we
     CHECK(resolve_mem(offsets, memkind));
     nulpa_graph *g = new nulpa_graph();
     memset(&g->stats, 0, sizeof g->stats);
-    if (const char *e = getenv("NULPA_WARP_KERNEL")) g->warp_kernel = atoi(e);
     g->n_rows = n_rows;
     g->n_global = n_global;
     g->row_begin = row_begin;
