@@ -76,18 +76,18 @@ def peaks():
 
 
 def algorithmic_bytes(st, b, weighted):
-    """Compulsory DRAM bytes of bin b over a run (DESIGN.md 'Kernels and
-    their rooflines'): per processed vertex 4 (bin list) + 16 (two offsets)
-    + 2 (flag read + clear) + 4 (own label); per scanned CSR entry 4 (index)
-    + 4 (weight, if stored); per changed vertex 4 (label write) and per CSR
-    entry of a changed vertex 4 (index re-read) + 1 (neighbour flag write).
-    Neighbour-label gathers are NOT counted (the label array is re-used
-    from cache); this is a lower bound on DRAM traffic."""
+    """Bytes Algorithm 1 moves for bin b over a run, each
+    array element counted once per use (DESIGN.md "Kernels and their
+    rooflines"): per processed vertex 4 (bin-list entry) + 16 (offsets O_i,
+    O_i+1) + 2 (flag read + clear) + 4 (own label C[i]); per scanned CSR entry
+    4 (index j) + 4 (weight, if stored) + 4 (neighbour label C[j], line 340);
+    per changed vertex 4 (label write) and 1 per CSR entry of a changed
+    vertex (mark j unprocessed, line 348)."""
     v = st["vertices_processed"][b]
     e = st["edges_scanned"][b]
     c = st["vertices_changed"][b]
     ce = st["changed_edges"][b]
-    return v * 26 + e * (8 if weighted else 4) + c * 4 + ce * 5
+    return v * 26 + e * (12 if weighted else 8) + c * 4 + ce * 1
 
 
 class Clocks:

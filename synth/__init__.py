@@ -63,13 +63,17 @@ def _gen(seed: int, device) -> torch.Generator:
     return g
 
 
+_CHUNK = 1 << 29   # elements per sort / unique call (CUB handles < 2^31)
+
+
 def from_edges(src: torch.Tensor, dst: torch.Tensor, N: int, *, weighted: bool = False,
                seed: int = 0, name: str = "graph", keep_self_loops: bool = False,
                truth: Optional[torch.Tensor] = None) -> Graph:
     """Build an undirected simple CSR graph from a list of (src, dst) pairs.
 
     Pairs are canonicalised to (min, max), deduplicated, optionally given one
-    weight each, then emitted in both directions and sorted by (src, dst)."""
+    weight each, then emitted in both directions and sorted by (src, dst).
+    Large inputs are processed in vertex-range buckets (sorts stay < 2^31)."""
     device = src.device
     src = src.to(torch.int64)
     dst = dst.to(torch.int64)
@@ -80,8 +84,21 @@ def from_edges(src: torch.Tensor, dst: torch.Tensor, N: int, *, weighted: bool =
     hi = torch.maximum(src, dst)
     del src, dst
     key = lo * N + hi
-    del lo, hi
-    key = torch.unique(key)                      # sorted, deduplicated undirected edges
+    del hi
+    nb = max(1, -(-key.numel() // _CHUNK))
+    if nb == 1:
+        del lo
+        key = torch.unique(key)                  # sorted, deduplicated undirected edges
+    else:
+        # bucket by the smaller endpoint: sorted order is preserved bucket by bucket
+        bucket = (lo * nb) // max(N, 1)
+        del lo
+        parts = []
+        for bk in range(nb):
+            parts.append(torch.unique(key[bucket == bk]))
+        del bucket, key
+        key = torch.cat(parts)
+        del parts
     u = key // N
     v = key - u * N
     del key
@@ -90,34 +107,35 @@ def from_edges(src: torch.Tensor, dst: torch.Tensor, N: int, *, weighted: bool =
         g = _gen(seed ^ 0x5EED, device)
         # float32 in (0, 1]: 1 - U[0,1)
         w_und = 1.0 - torch.rand(u.numel(), generator=g, device=device, dtype=torch.float32)
-    loop = u == v
-    if bool(loop.any()):
-        # a self-loop is stored once (it is its own reverse)
-        nl = ~loop
-        s_all = torch.cat([u, v[nl]])
-        d_all = torch.cat([v, u[nl]])
-        w_all = None if w_und is None else torch.cat([w_und, w_und[nl]])
-    else:
-        s_all = torch.cat([u, v])
-        d_all = torch.cat([v, u])
-        w_all = None if w_und is None else torch.cat([w_und, w_und])
+    # directed entries, bucketed by source vertex range
+    m_dir = 2 * u.numel()
+    nbd = max(1, -(-m_dir // _CHUNK))
+    ind_parts, w_parts = [], []
+    counts = torch.zeros(N, dtype=torch.int64, device=device)
+    for bk in range(nbd):
+        a0, a1 = (N * bk) // nbd, (N * (bk + 1)) // nbd
+        mu = (u >= a0) & (u < a1)
+        mv = (v >= a0) & (v < a1) & (u != v)          # a self-loop is stored once
+        s_b = torch.cat([u[mu], v[mv]])
+        d_b = torch.cat([v[mu], u[mv]])
+        w_b = None if w_und is None else torch.cat([w_und[mu], w_und[mv]])
+        del mu, mv
+        dkey = s_b * N + d_b
+        del d_b
+        if w_b is None:
+            dkey, _ = torch.sort(dkey)
+        else:
+            dkey, perm = torch.sort(dkey)
+            w_parts.append(w_b[perm])
+            del perm, w_b
+        srt_s = dkey // N
+        ind_parts.append((dkey - srt_s * N).to(torch.int32))
+        counts += torch.bincount(srt_s, minlength=N)
+        del dkey, srt_s, s_b
     del u, v, w_und
-    dkey = s_all * N + d_all
-    del d_all
-    if w_all is None:
-        dkey, _ = torch.sort(dkey)
-        srt_s = dkey // N
-        indices = (dkey - srt_s * N).to(torch.int32)
-        weights = None
-    else:
-        dkey, perm = torch.sort(dkey)
-        srt_s = dkey // N
-        indices = (dkey - srt_s * N).to(torch.int32)
-        weights = w_all[perm]
-        del perm, w_all
-    del dkey, s_all
-    counts = torch.bincount(srt_s, minlength=N)
-    del srt_s
+    indices = torch.cat(ind_parts) if len(ind_parts) > 1 else ind_parts[0]
+    weights = None if not w_parts else (torch.cat(w_parts) if len(w_parts) > 1 else w_parts[0])
+    del ind_parts, w_parts
     offsets = torch.zeros(N + 1, dtype=torch.int64, device=device)
     torch.cumsum(counts, 0, out=offsets[1:])
     return Graph(offsets, indices, weights, name, truth)
@@ -312,7 +330,7 @@ def kmer(n: int = 1_000_000, branch: float = 0.05, *, seed: int = 0, device="cpu
     return from_edges(torch.cat([a, xa]), torch.cat([b, xb]), n, weighted=weighted, seed=seed, name="kmer")
 
 
-def web(n: int = 40_000_000, avg_out: float = 42.0, p_local: float = 0.95, gamma: float = 3.6,
+def web(n: int = 40_000_000, avg_out: float = 58.0, p_local: float = 0.95, gamma: float = 3.6,
         host_alpha: float = 1.4, host_min: int = 16, host_max: int = 400_000, max_out: int = 20_000, *,
         locality: str = "loguniform", global_target: str = "page", seed: int = 0, device="cpu",
         weighted: bool = False,

@@ -288,3 +288,55 @@ def test_invalid_params_raise():
         gg.run(block_degree=300)
     with pytest.raises(nl.NulpaError):
         gg.run(max_iterations=100)
+
+
+# ---------------------------------------------------------------------------
+# shard handles (multi-GPU mode) on one GPU: in synchronous mode the
+# bulk-synchronous shard protocol IS a global Jacobi sweep, so P shards
+# exchanging labels / flags after every sweep must reproduce the oracle's
+# synchronous run exactly (unit weights)
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("gname", ["sbm", "web", "hub", "road"])
+@pytest.mark.parametrize("world", [2, 3])
+def test_shards_sync_equal_oracle(gname, world):
+    from paper_conf_ipps_sahunk25_b200 import distributed as D
+    g = GRAPHS[gname](False)
+    C, it, dn = oracle.lpa(host(g), sync=True)
+    runners = []
+    for r in range(world):
+        sh = D.shard_graph(g.offsets, g.indices, None, r, world)
+        runners.append(D.CudaShardRunner(sh, mode=nl.SYNC, switch_degree=4, block_degree=12, giant_degree=40))
+    bounds = runners[0].shard.bounds
+    for run in runners:
+        run.reset()
+        b, e = run.row_begin, run.row_end
+        run.flags[:b].zero_()
+        run.flags[e:].zero_()
+    changed = []
+    for l in range(20):
+        pl = l % 4 == 0
+        d = sum(run.sweep(pl) for run in runners)
+        for q, (qb, qe) in enumerate(bounds):          # all-gather of labels
+            for run in runners:
+                run.labels[qb:qe].copy_(runners[q].labels[qb:qe])
+        F = torch.stack([run.flags for run in runners]).max(0).values   # all-reduce MAX
+        for run in runners:
+            run.flags.copy_(F)
+            run.flags[:run.row_begin].zero_()
+            run.flags[run.row_end:].zero_()
+        changed.append(d)
+        if not pl and d / g.N < 0.05:
+            break
+    assert changed == list(dn) and len(changed) == it
+    for run in runners:
+        np.testing.assert_array_equal(run.labels.cpu().numpy(), C)
+    # sharded modularity pieces add up to the whole-graph value
+    Sigma = torch.zeros(g.N, dtype=torch.float64, device="cuda")
+    sig = m2 = 0.0
+    for run in runners:
+        s_, m_ = run.modularity_partial(Sigma)
+        sig += s_
+        m2 += m_
+    q = runners[0].modularity_finish(Sigma, sig, m2)
+    assert abs(q - oracle.modularity(host(g), C)) < 1e-9
