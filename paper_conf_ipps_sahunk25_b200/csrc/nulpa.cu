@@ -576,6 +576,11 @@ __global__ void __launch_bounds__(kWarpThreads, 6) k_warp(SweepArgs a, const int
             auto fold = [&](int32_t key, float w, unsigned &grp) -> float {
                 grp = __match_any_sync(0xFFFFFFFFu, key);
                 if (W) {
+                    // all weights of the batch equal (e.g. the paper's default
+                    // weight 1): the group total is count * w, the correctly
+                    // rounded sum (exact for integer-valued weights)
+                    const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
+                    if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
                     const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
                     return maxn > 1 ? group_sum(grp, w, maxn) : w;
                 }
@@ -650,85 +655,139 @@ __global__ void __launch_bounds__(kWarpThreads, 6) k_warp(SweepArgs a, const int
 }
 
 // ---------------------------------------------------------------------------
-// block-per-vertex kernel: one CTA per vertex, table (p1 <= 4095) in dynamic
-// shared memory, persistent grid-stride over the bin.  PAPER.md:243.
+// block-per-vertex kernel: one CTA of 4 warps per vertex, the
+// vertex's table -- p1 = nextPow2(D)-1 slots as in PAPER.md:208, <= 4095 --
+// in shared memory, cleared at the start of each vertex.  Each warp folds its
+// 32-edge batches (match_any groups); a group leader claims the label's slot
+// (Algorithm 2 probing, atomicCAS) and adds the group total with one
+// atomicAdd, whose return value gives the label's running total, so the
+// maximum over all leaders' totals is hashtableMaxKey (no table scan).
 // ---------------------------------------------------------------------------
+constexpr int kBlkThreads = 128;
+
 template <bool SYNC, bool W, int TIE>
-__global__ void __launch_bounds__(kBlockThreads) k_block(SweepArgs a, const int32_t *__restrict__ list,
-                                                         int64_t n) {
+__global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_t *__restrict__ list,
+                                                        int64_t n) {
     extern __shared__ int32_t dyn[];
     int32_t *Hk = dyn;
     float *Hv = reinterpret_cast<float *>(dyn + kBlockCap);
-    __shared__ uint64_t red[kBlockThreads / 32];
-    __shared__ int s_act;
+    __shared__ int64_t m_o[32];
+    __shared__ int32_t m_r[32], m_d[32], m_ci[32];
+    __shared__ unsigned s_act;
     __shared__ int s_changed;
+    __shared__ uint32_t s_bw[kBlkThreads / 32], s_rr[kBlkThreads / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int s = threadIdx.x; s < kBlockCap; s += kBlockThreads) {
-        Hk[s] = kEmpty;
-        Hv[s] = 0.0f;
-    }
     unsigned long long n_act = 0, n_edges = 0, n_changed = 0, n_changed_edges = 0;
-    __syncthreads();
-    for (int64_t t = blockIdx.x; t < n; t += gridDim.x) {
-        int32_t r = list[t];
-        int64_t v = r + a.row_begin;
-        if (threadIdx.x == 0) {
-            int f = a.flag_in[v];
-            s_act = f;
-            if (f && !SYNC) a.flag_in[v] = 0;
+    const int64_t ngroups = (n + 31) / 32;
+    for (int64_t gq = blockIdx.x; gq < ngroups; gq += gridDim.x) {
+        // metadata of 32 consecutive bin entries in one round trip (warp 0)
+        if (wid == 0) {
+            const int64_t t = gq * 32 + lane;
+            int f = 0;
+            if (t < n) {
+                const int32_t r = list[t];
+                const int64_t v = r + a.row_begin;
+                f = a.flag_in[v];
+                m_r[lane] = r;
+                if (f) {
+                    const int64_t o = a.offsets[r];
+                    m_o[lane] = o;
+                    m_d[lane] = (int32_t)(a.offsets[r + 1] - o);
+                    m_ci[lane] = a.lab_in[v];
+                    if (!SYNC) a.flag_in[v] = 0;           // mark i as processed
+                }
+            }
+            const unsigned am = __ballot_sync(0xFFFFFFFFu, f != 0);
+            if (lane == 0) s_act = am;
         }
         __syncthreads();
-        if (s_act) {
-            int64_t o = a.offsets[r];
-            uint32_t deg = (uint32_t)(a.offsets[r + 1] - o);
+        unsigned act = s_act;
+        while (act) {
+            const int k = __ffs(act) - 1;
+            act &= act - 1;
+            const int64_t o = m_o[k];
+            const uint32_t deg = (uint32_t)m_d[k];
+            const int64_t v = m_r[k] + a.row_begin;
             Hash h;
             h.init(deg);
-            for (uint32_t b = (uint32_t)wid * 32; b < deg; b += kBlockThreads) {
-                int32_t key = kEmpty;
-                float w = 0.0f;
-                if (b + lane < deg) {
-                    const int32_t j = a.indices[o + b + lane];
-                    if (j != (int32_t)v) {
-                        key = a.lab_in[j];
-                        if (W) w = a.weights[o + b + lane];
-                    }
-                }
-                warp_batch_accumulate_atomic<W>(Hk, Hv, h, key, w);
+            for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {   // hashtableClear
+                Hk[q] = kEmpty;
+                Hv[q] = 0.0f;
             }
             __syncthreads();
             TieOrder<TIE> to;
             to.init(h);
-            uint64_t best = 0;
-            for (uint32_t s = threadIdx.x; s < h.p1; s += kBlockThreads) {
-                int32_t k = Hk[s];
-                if (k != kEmpty) {
-                    uint64_t c = pack_cand(Hv[s], k, to);
-                    best = c > best ? c : best;
-                    Hk[s] = kEmpty;
-                    Hv[s] = 0.0f;
+            uint32_t bw = 0;
+            int32_t bk = 0;
+            auto fold = [&](int32_t key, float w) {
+                const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+                float x;
+                if (W) {
+                    const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
+                    if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) {
+                        x = (float)__popc(grp) * w;
+                    } else {
+                        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+                        x = maxn > 1 ? group_sum(grp, w, maxn) : w;
+                    }
+                } else {
+                    x = (float)__popc(grp);
                 }
+                if (key != kEmpty && lane == __ffs(grp) - 1) {
+                    const uint32_t slot = ht_claim(Hk, h, key);
+                    const float V = __fadd_rn(atomicAdd(&Hv[slot], x), x);
+                    const uint32_t vb = __float_as_uint(V) + 1;
+                    if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
+                        bw = vb;
+                        bk = key;
+                    }
+                }
+            };
+            // two 32-edge batches per warp per step: both index loads, then
+            // both label gathers in flight together
+            for (uint32_t b = (uint32_t)wid * 32; b < deg; b += 2 * kBlkThreads) {
+                const uint32_t e0 = b + lane, e1 = b + kBlkThreads + lane;
+                const int32_t j0 = e0 < deg ? a.indices[o + e0] : -1;
+                const int32_t j1 = e1 < deg ? a.indices[o + e1] : -1;
+                float w0 = 0.0f, w1 = 0.0f;
+                if (W) {
+                    if (e0 < deg) w0 = a.weights[o + e0];
+                    if (e1 < deg) w1 = a.weights[o + e1];
+                }
+                const int32_t k0 = (j0 >= 0 && j0 != (int32_t)v) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
+                const int32_t k1 = (j1 >= 0 && j1 != (int32_t)v) ? a.lab_in[j1] : kEmpty;
+                fold(k0, w0);
+                if (b + kBlkThreads < deg) fold(k1, w1);
             }
-            best = warp_max_u64(best);
-            if (lane == 0) red[wid] = best;
+            // hashtableMaxKey over the 4 warps
+            const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
+            const uint32_t rr = (bw == W1 && W1) ? 0xFFFFFFFFu - to.rank(bk) : 0u;
+            const uint32_t R1 = __reduce_max_sync(0xFFFFFFFFu, rr);
+            if (lane == 0) {
+                s_bw[wid] = W1;
+                s_rr[wid] = R1;
+            }
             __syncthreads();
-            if (wid == 0) {
-                uint64_t b = lane < kBlockThreads / 32 ? red[lane] : 0;
-                b = warp_max_u64(b);
-                if (lane == 0) {
-                    int32_t ci = a.lab_in[v];
-                    int32_t cs = b ? cand_label(b, to) : kEmpty;
-                    int ch = accept_move(cs, ci, a.pickless);
-                    if (ch) a.lab_out[v] = cs;
-                    s_changed = ch;
-                    n_act += 1;
-                    n_edges += deg;
-                    n_changed += ch;
-                    n_changed_edges += ch ? deg : 0;
+            if (threadIdx.x == 0) {
+                uint32_t Wb = 0, Rb = 0;
+                for (int q = 0; q < kBlkThreads / 32; ++q) {
+                    if (s_bw[q] > Wb || (s_bw[q] == Wb && s_rr[q] > Rb)) {
+                        Wb = s_bw[q];
+                        Rb = s_rr[q];
+                    }
                 }
+                const int32_t cs = Wb ? to.unrank(0xFFFFFFFFu - Rb) : kEmpty;
+                const int ch = accept_move(cs, m_ci[k], a.pickless);
+                if (ch) a.lab_out[v] = cs;
+                s_changed = ch;
+                n_act += 1;
+                n_edges += deg;
+                n_changed += ch;
+                n_changed_edges += ch ? deg : 0;
             }
             __syncthreads();
             if (s_changed)
-                for (int64_t e = o + threadIdx.x; e < o + deg; e += kBlockThreads) a.flag_out[a.indices[e]] = 1;
+                for (uint32_t b = threadIdx.x; b < deg; b += kBlkThreads) a.flag_out[a.indices[o + b]] = 1;
         }
         __syncthreads();
     }
@@ -896,12 +955,14 @@ __device__ __forceinline__ int bin_of(int64_t d, int32_t t1, int32_t t2, int32_t
 }
 
 __global__ void __launch_bounds__(kBinTile) k_bin_count(const int64_t *offsets, int64_t n, int32_t t1, int32_t t2,
-                                                        int32_t t3, int64_t *counts, unsigned long long *edges) {
+                                                        int32_t t3, int64_t *counts, unsigned long long *edges,
+                                                        unsigned long long *maxdeg) {
     __shared__ int64_t c[4];
-    __shared__ unsigned long long ed[4];
+    __shared__ unsigned long long ed[4], md[4];
     if (threadIdx.x < 4) {
         c[threadIdx.x] = 0;
         ed[threadIdx.x] = 0;
+        md[threadIdx.x] = 0;
     }
     __syncthreads();
     for (int k = 0; k < kBinTiles; ++k) {
@@ -912,6 +973,7 @@ __global__ void __launch_bounds__(kBinTile) k_bin_count(const int64_t *offsets, 
             if (b >= 0) {
                 atomicAdd((unsigned long long *)&c[b], 1ull);
                 atomicAdd(&ed[b], (unsigned long long)d);
+                atomicMax(&md[b], (unsigned long long)d);
             }
         }
     }
@@ -919,6 +981,7 @@ __global__ void __launch_bounds__(kBinTile) k_bin_count(const int64_t *offsets, 
     if (threadIdx.x < 4) {
         counts[(int64_t)blockIdx.x * 4 + threadIdx.x] = c[threadIdx.x];
         atomicAdd(&edges[threadIdx.x], ed[threadIdx.x]);
+        atomicMax(&maxdeg[threadIdx.x], md[threadIdx.x]);
     }
 }
 
@@ -1110,6 +1173,7 @@ struct nulpa_graph {
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
     int64_t bin_n[4] = {0, 0, 0, 0};
     int64_t bin_e[4] = {0, 0, 0, 0};
+    int64_t bin_maxdeg[4] = {0, 0, 0, 0};
     // giant
     int64_t n_chunks = 0;
     int32_t *chunk_g = nullptr;
@@ -1192,10 +1256,10 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
     unsigned long long *edges = nullptr;
     CHECK(dalloc(&counts, (size_t)std::max<int64_t>(nb, 1) * 4));
     CHECK(dalloc(&totals, 4));
-    CHECK(dalloc(&edges, 4));
-    CU(cudaMemsetAsync(edges, 0, 4 * sizeof(unsigned long long), g->stream));
+    CHECK(dalloc(&edges, 8));
+    CU(cudaMemsetAsync(edges, 0, 8 * sizeof(unsigned long long), g->stream));
     if (nb > 0) {
-        k_bin_count<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, edges);
+        k_bin_count<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, edges, edges + 4);
         CU(cudaGetLastError());
         k_bin_scan<<<1, 1024, 0, g->stream>>>(counts, nb, totals);
         CU(cudaGetLastError());
@@ -1203,7 +1267,7 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CU(cudaMemsetAsync(totals, 0, 4 * sizeof(int64_t), g->stream));
     }
     int64_t ht[4];
-    unsigned long long he[4];
+    unsigned long long he[8];
     CU(cudaMemcpyAsync(ht, totals, sizeof ht, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaMemcpyAsync(he, edges, sizeof he, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
@@ -1211,6 +1275,7 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
     for (int b = 0; b < 4; ++b) {
         g->bin_n[b] = ht[b];
         g->bin_e[b] = (int64_t)he[b];
+        g->bin_maxdeg[b] = (int64_t)he[4 + b];
         CHECK(dalloc(&g->bin_list[b], (size_t)ht[b]));
         L.l[b] = g->bin_list[b];
     }
@@ -1301,11 +1366,12 @@ template <bool SYNC, bool W, int TIE>
 int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const int64_t n = g->bin_n[0];
     const int grid = grid_for(n, kThreadThreads);
-    if (g->t1 <= 5)
+    const int64_t md = g->bin_maxdeg[0];     // register table sized by the bin's largest degree
+    if (md <= 4)
         k_thread<SYNC, W, TIE, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    else if (g->t1 <= 9)
+    else if (md <= 8)
         k_thread<SYNC, W, TIE, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    else if (g->t1 <= 17)
+    else if (md <= 16)
         k_thread<SYNC, W, TIE, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else
         k_thread<SYNC, W, TIE, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
@@ -1377,7 +1443,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(2, 0));
         if (n > 0) {
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W, TIE><<<grid_for(n, 1, sms * 4), kBlockThreads, smem, g->stream>>>(a, g->bin_list[2], n);
+            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, g->stream>>>(a, g->bin_list[2], n);
             CU(cudaGetLastError());
             g->stats.launches[2] += 1;
         }
@@ -1489,7 +1555,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->mode = NULPA_ASYNC;
     p->switch_degree = 16;
     p->block_degree = 256;
-    p->giant_degree = 4096;
+    p->giant_degree = 2048;
     p->reset = 1;
     p->timing = 0;
     p->tie_rule = NULPA_TIE_SMALLEST;
