@@ -373,6 +373,9 @@ __device__ __forceinline__ bool accept_move(int32_t cstar, int32_t ci, int pickl
     return cstar != kEmpty && cstar != ci && (!pickless || cstar <= ci);
 }
 
+// CSR indices / weights are streamed once per sweep: they are loaded with
+// __ldcs (ld.global.cs, evict-first) so they do not push the label and flag
+// vectors -- the gathered, reused data -- out of L1/L2.
 struct SweepArgs {
     const int64_t *__restrict__ offsets;
     const int32_t *__restrict__ indices;
@@ -551,12 +554,12 @@ __global__ void __launch_bounds__(kWarpThreads, 6) k_warp(SweepArgs a, const int
             // the first 64 entries of the row stay in registers; indices and
             // weights first, then all the neighbour labels
             const bool v0 = (uint32_t)lane < dk, v1 = (uint32_t)(lane + 32) < dk;
-            const int32_t j0 = v0 ? a.indices[ok + lane] : -1;
-            const int32_t j1 = v1 ? a.indices[ok + 32 + lane] : -1;
+            const int32_t j0 = v0 ? __ldcs(a.indices + ok + lane) : -1;
+            const int32_t j1 = v1 ? __ldcs(a.indices + ok + 32 + lane) : -1;
             float w0 = 0.0f, w1 = 0.0f;
             if (W) {
-                if (v0) w0 = a.weights[ok + lane];
-                if (v1) w1 = a.weights[ok + 32 + lane];
+                if (v0) w0 = __ldcs(a.weights + ok + lane);
+                if (v1) w1 = __ldcs(a.weights + ok + 32 + lane);
             }
             const int32_t k0 = (j0 >= 0 && j0 != (int32_t)vk) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
             const int32_t k1 = (j1 >= 0 && j1 != (int32_t)vk) ? a.lab_in[j1] : kEmpty;
@@ -603,12 +606,12 @@ __global__ void __launch_bounds__(kWarpThreads, 6) k_warp(SweepArgs a, const int
                 batch(k1, w1);
                 for (uint32_t b = 64; b < dk; b += 64) {
                     const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
-                    const int32_t i0 = u0 ? a.indices[ok + b + lane] : -1;
-                    const int32_t i1 = u1 ? a.indices[ok + b + 32 + lane] : -1;
+                    const int32_t i0 = u0 ? __ldcs(a.indices + ok + b + lane) : -1;
+                    const int32_t i1 = u1 ? __ldcs(a.indices + ok + b + 32 + lane) : -1;
                     float x0 = 0.0f, x1 = 0.0f;
                     if (W) {
-                        if (u0) x0 = a.weights[ok + b + lane];
-                        if (u1) x1 = a.weights[ok + b + 32 + lane];
+                        if (u0) x0 = __ldcs(a.weights + ok + b + lane);
+                        if (u1) x1 = __ldcs(a.weights + ok + b + 32 + lane);
                     }
                     const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
                     const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
@@ -747,12 +750,12 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_
             // both label gathers in flight together
             for (uint32_t b = (uint32_t)wid * 32; b < deg; b += 2 * kBlkThreads) {
                 const uint32_t e0 = b + lane, e1 = b + kBlkThreads + lane;
-                const int32_t j0 = e0 < deg ? a.indices[o + e0] : -1;
-                const int32_t j1 = e1 < deg ? a.indices[o + e1] : -1;
+                const int32_t j0 = e0 < deg ? __ldcs(a.indices + o + e0) : -1;
+                const int32_t j1 = e1 < deg ? __ldcs(a.indices + o + e1) : -1;
                 float w0 = 0.0f, w1 = 0.0f;
                 if (W) {
-                    if (e0 < deg) w0 = a.weights[o + e0];
-                    if (e1 < deg) w1 = a.weights[o + e1];
+                    if (e0 < deg) w0 = __ldcs(a.weights + o + e0);
+                    if (e1 < deg) w1 = __ldcs(a.weights + o + e1);
                 }
                 const int32_t k0 = (j0 >= 0 && j0 != (int32_t)v) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
                 const int32_t k1 = (j1 >= 0 && j1 != (int32_t)v) ? a.lab_in[j1] : kEmpty;
@@ -858,10 +861,10 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
         int32_t key = kEmpty;
         float w = 0.0f;
         if (b + lane < e1) {
-            const int32_t j = a.indices[b + lane];
+            const int32_t j = __ldcs(a.indices + b + lane);
             if (j != (int32_t)v) {
                 key = a.lab_in[j];
-                if (W) w = a.weights[b + lane];
+                if (W) w = __ldcs(a.weights + b + lane);
             }
         }
         warp_batch_accumulate_atomic<W>(Hk, Hv, hc, key, w);
