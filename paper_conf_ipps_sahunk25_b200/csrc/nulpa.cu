@@ -15,7 +15,7 @@
 //
 // Kernels of one sweep (lpaMove), launched on the handle's stream in order
 // giant -> block -> warp -> thread (largest work first):
-//   k_giant_snapshot / k_giant_accumulate / k_giant_finalize / k_giant_mark
+//   k_giant_snapshot / k_giant_accumulate / k_giant_reduce / k_giant_decide / k_giant_mark
 //   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
 //   k_warp    one warp per vertex, shared-memory table (<= 255 slots)
 //   k_thread  one thread per vertex, labels in registers (degree < 32)
@@ -41,6 +41,10 @@ constexpr int kCtr = 24;                 // counters per iteration
 
 constexpr int kWarpThreads = 256;        // k_warp: 8 warps per CTA
 constexpr int kWarpTab = 256;            // slots of a k_warp table (P1 = 255)
+#ifndef NULPA_WARP_CTAS
+#define NULPA_WARP_CTAS 6
+#endif
+constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;  // resident k_warp CTAs per SM (register budget)
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
 constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
 constexpr int kGiantChunk = 4096;        // edges per giant chunk
@@ -266,12 +270,12 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
 // value update is a plain read-modify-write; only the slot claim is atomic
 // (64-bit shared-memory CAS).
 template <uint32_t P1>
-__device__ __noinline__ float tt_add_slow(uint64_t *tk, float *tv, uint32_t tag, int32_t k, float x) {
+__device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, int32_t k, float x) {
     constexpr uint32_t p1 = P1, p2 = 2 * P1 + 1;
     const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
     uint32_t i = (uint32_t)k % p1;
     uint32_t di = 1;
-    const uint32_t km = ((uint32_t)k % p2) % p1;           // k mod p2 (2nd hash)
+    uint32_t km = 0xFFFFFFFFu;                             // k mod p2, computed on the first collision
     for (int t = 0;; ++t) {
         const uint64_t cur = *((volatile uint64_t *)&tk[i]);
         if (cur == want) {
@@ -288,6 +292,7 @@ __device__ __noinline__ float tt_add_slow(uint64_t *tk, float *tv, uint32_t tag,
             }
         }
         if (t < kMaxRetries) {
+            if (km == 0xFFFFFFFFu) km = ((uint32_t)k % p2) % p1;
             i += di;
             if (i >= p1) i -= p1;
             di = 2 * di + km;
@@ -299,32 +304,37 @@ __device__ __noinline__ float tt_add_slow(uint64_t *tk, float *tv, uint32_t tag,
     }
 }
 
-// Fast path: the home slot k mod p1 either holds (tag, k) or is free (a
-// stale tag) and is claimed; anything else (a collision, or a lost claim
-// race) restarts the full probe sequence out of line.
-template <uint32_t P1>
-__device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, int32_t k, float x) {
-    const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
-    const uint32_t i = (uint32_t)k % P1;
-    const uint64_t cur = tk[i];
-    if (cur == want) {
-        const float V = __fadd_rn(tv[i], x);
-        tv[i] = V;
-        return V;
+// One 32-edge batch of a warp against the warp's PRIVATE table: lanes
+// holding the same label (match_any) are folded onto their lowest lane (the
+// leader), which claims the label's slot (Algorithm 2 probing, atomicCAS on
+// the key) and adds the group's weight with a plain shared-memory
+// read-modify-write -- no other lane of the batch touches that slot, and
+// batches are ordered by __syncwarp, so no float atomics are needed (the GPU
+// has no native shared-memory float atomicAdd).  Unit weights: the group
+// weight is the member count, exact.  key == kEmpty marks an idle lane.
+template <bool W>
+__device__ __forceinline__ void warp_batch_accumulate(int32_t *Hk, float *Hv, const Hash &h, int32_t key, float w) {
+    const int lane = threadIdx.x & 31;
+    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+    const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
+    float sum;
+    if (W) {
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
+    } else {
+        sum = (float)__popc(grp);
     }
-    if ((uint32_t)(cur >> 32) != tag &&
-        atomicCAS((unsigned long long *)&tk[i], (unsigned long long)cur, (unsigned long long)want) == cur) {
-        tv[i] = x;
-        return x;
+    if (leader) {
+        const uint32_t slot = ht_claim(Hk, h, key);
+        Hv[slot] = __fadd_rn(Hv[slot], sum);
     }
-    return tt_add_slow<P1>(tk, tv, tag, k, x);
+    __syncwarp();
 }
 
-// One 32-edge batch of a warp against a table shared by several warps (giant
-// chunk tables): lanes holding the same label (match_any) are folded onto
-// their lowest lane, which claims the label's slot (Algorithm 2 probing,
-// atomicCAS) and adds the group total with one shared-memory atomicAdd (a
-// CAS loop on this GPU, contended by at most one lane per warp and label).
+// The same folding for a table shared by several warps (block / giant
+// kernels): the leader adds its group's sum with one shared-memory
+// atomicAdd (a CAS loop on this GPU, now contended by at most one lane per
+// warp and label).
 template <bool W>
 __device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float *Hv, const Hash &h, int32_t key,
                                                              float w) {
@@ -333,13 +343,8 @@ __device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float 
     const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
     float sum;
     if (W) {
-        const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
-        if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) {
-            sum = (float)__popc(grp) * w;
-        } else {
-            const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-            sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
-        }
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
     } else {
         sum = (float)__popc(grp);
     }
@@ -487,40 +492,15 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
 // warp-per-vertex kernel: one 32-lane warp per vertex, the vertex's table
 // (p1 <= 255 slots) in shared memory, persistent grid-stride over the bin.
 // ---------------------------------------------------------------------------
-// Peel test for a 64-entry row (two 32-lane batches k0 / k1): at most
-// kPeelMax distinct labels in total (leaders of both batches' match_any
-// groups) and, when weights are stored, all weights equal.
-constexpr int kPeelMax = 8;
-__device__ __forceinline__ bool peel_ok(int32_t k0, int32_t k1, float w0, float w1) {
-    const int lane = threadIdx.x & 31;
-    const unsigned g0 = __match_any_sync(0xFFFFFFFFu, k0);
-    const unsigned g1 = __match_any_sync(0xFFFFFFFFu, k1);
-    const unsigned l0 = __ballot_sync(0xFFFFFFFFu, k0 != kEmpty && lane == __ffs(g0) - 1);
-    const unsigned l1 = __ballot_sync(0xFFFFFFFFu, k1 != kEmpty && lane == __ffs(g1) - 1);
-    if (__popc(l0) + __popc(l1) > kPeelMax) return false;
-    const unsigned any0 = __ballot_sync(0xFFFFFFFFu, k0 != kEmpty);
-    const unsigned any1 = __ballot_sync(0xFFFFFFFFu, k1 != kEmpty);
-    if (!(any0 | any1)) return true;
-    const int src = any0 ? __ffs(any0) - 1 : __ffs(any1) - 1;
-    const float wr = __shfl_sync(0xFFFFFFFFu, any0 ? w0 : w1, src);
-    return __all_sync(0xFFFFFFFFu, (k0 == kEmpty || w0 == wr) && (k1 == kEmpty || w1 == wr));
-}
-
-// Per-warp shared memory of k_warp: the tagged table.
-struct WarpSmem {
-    uint64_t tk[kWarpTab];
-    float tv[kWarpTab];
-};
-
 template <bool SYNC, bool W, int TIE>
-__global__ void __launch_bounds__(kWarpThreads, 4) k_warp(SweepArgs a, const int32_t *__restrict__ list,
+__global__ void __launch_bounds__(kWarpThreads, kWarpCtasPerSm) k_warp(SweepArgs a, const int32_t *__restrict__ list,
                                                           int64_t n) {
-    extern __shared__ __align__(16) unsigned char wsm[];
+    __shared__ uint64_t s_tk[kWarpThreads / 32][kWarpTab];   // static: 32-bit shared addressing
+    __shared__ float s_tv[kWarpThreads / 32][kWarpTab];
     __shared__ unsigned long long bctr[4];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    WarpSmem &S = reinterpret_cast<WarpSmem *>(wsm)[wid];
-    uint64_t *tk = S.tk;
-    float *tv = S.tv;
+    uint64_t *tk = s_tk[wid];
+    float *tv = s_tv[wid];
     for (int q = lane; q < kWarpTab; q += 32) tk[q] = 0;   // tag 0: empty for every vertex
     if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
     __syncthreads();
@@ -548,130 +528,104 @@ __global__ void __launch_bounds__(kWarpThreads, 4) k_warp(SweepArgs a, const int
             if (!SYNC) a.flag_in[r + a.row_begin] = 0;     // mark i as processed
         }
         unsigned act = __ballot_sync(0xFFFFFFFFu, f != 0);
-        // Active vertices are taken TWO at a time: both rows' index loads,
-        // then both rows' label gathers, are issued before either vertex is
-        // folded, so each global round trip is shared by two vertices (ILP 2
-        // against the long-scoreboard stalls that dominate this kernel).
         while (act) {
-            int ks[2];
-            ks[0] = __ffs(act) - 1;
+            const int k = __ffs(act) - 1;
             act &= act - 1;
-            const bool two = act != 0;
-            ks[1] = two ? __ffs(act) - 1 : ks[0];
-            if (two) act &= act - 1;
-            int64_t ok[2], vk[2];
-            uint32_t dk[2];
-            int32_t cik[2], j0[2], j1[2], k0[2], k1[2];
-            float w0[2], w1[2];
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                const int k = ks[u];
-                vk[u] = (int64_t)__shfl_sync(0xFFFFFFFFu, r, k) + a.row_begin;
-                ok[u] = __shfl_sync(0xFFFFFFFFu, o, k);
-                dk[u] = __shfl_sync(0xFFFFFFFFu, deg, k);
-                cik[u] = __shfl_sync(0xFFFFFFFFu, ci, k);
+            const int32_t rk = __shfl_sync(0xFFFFFFFFu, r, k);
+            const int64_t ok = __shfl_sync(0xFFFFFFFFu, o, k);
+            const uint32_t dk = __shfl_sync(0xFFFFFFFFu, deg, k);
+            const int32_t cik = __shfl_sync(0xFFFFFFFFu, ci, k);
+            const int64_t vk = rk + a.row_begin;
+            Hash h;
+            h.init(dk);
+            TieOrder<TIE> to;
+            to.init(h);
+            // the first 64 entries of the row stay in registers; indices and
+            // weights first, then all the neighbour labels
+            const bool v0 = (uint32_t)lane < dk, v1 = (uint32_t)(lane + 32) < dk;
+            const int32_t j0 = v0 ? __ldcs(a.indices + ok + lane) : -1;
+            const int32_t j1 = v1 ? __ldcs(a.indices + ok + 32 + lane) : -1;
+            float w0 = 0.0f, w1 = 0.0f;
+            if (W) {
+                if (v0) w0 = __ldcs(a.weights + ok + lane);
+                if (v1) w1 = __ldcs(a.weights + ok + 32 + lane);
             }
-            if (!two) dk[1] = 0;
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                const bool v0 = (uint32_t)lane < dk[u], v1 = (uint32_t)(lane + 32) < dk[u];
-                j0[u] = v0 ? __ldcs(a.indices + ok[u] + lane) : -1;
-                j1[u] = v1 ? __ldcs(a.indices + ok[u] + 32 + lane) : -1;
-                w0[u] = 0.0f;
-                w1[u] = 0.0f;
+            const int32_t k0 = (j0 >= 0 && j0 != (int32_t)vk) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
+            const int32_t k1 = (j1 >= 0 && j1 != (int32_t)vk) ? a.lab_in[j1] : kEmpty;
+            // per-lane running best (weight bits + 1, label) over the label
+            // totals this lane produced as a group leader; the maximum over
+            // all lanes is hashtableMaxKey (totals only grow, so partial
+            // totals never exceed the final maximum)
+            uint32_t bw = 0;
+            int32_t bk = 0;
+            auto offer = [&](float V, int32_t key) {
+                const uint32_t vb = __float_as_uint(V) + 1;
+                if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
+                    bw = vb;
+                    bk = key;
+                }
+            };
+            auto fold = [&](int32_t key, float w, unsigned &grp) -> float {
+                grp = __match_any_sync(0xFFFFFFFFu, key);
                 if (W) {
-                    if (v0) w0[u] = __ldcs(a.weights + ok[u] + lane);
-                    if (v1) w1[u] = __ldcs(a.weights + ok[u] + 32 + lane);
+                    // all weights of the batch equal (e.g. the paper's default
+                    // weight 1): the group total is count * w, the correctly
+                    // rounded sum (exact for integer-valued weights)
+                    const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
+                    if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
+                    const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+                    return maxn > 1 ? group_sum(grp, w, maxn) : w;
                 }
-            }
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                k0[u] = (j0[u] >= 0 && j0[u] != (int32_t)vk[u]) ? a.lab_in[j0[u]] : kEmpty;   // "if j = i continue"
-                k1[u] = (j1[u] >= 0 && j1[u] != (int32_t)vk[u]) ? a.lab_in[j1[u]] : kEmpty;
-            }
-#pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                if (u == 1 && !two) break;
-                Hash h;
-                h.init(dk[u]);
-                TieOrder<TIE> to;
-                to.init(h);
-                // per-lane running best (weight bits + 1, label) over the label
-                // totals this lane produced as a group leader; the maximum over
-                // all lanes is hashtableMaxKey (totals only grow, so partial
-                // totals never exceed the final maximum)
-                uint32_t bw = 0;
-                int32_t bk = 0;
-                auto offer = [&](float V, int32_t key) {
-                    const uint32_t vb = __float_as_uint(V) + 1;
-                    if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
-                        bw = vb;
-                        bk = key;
-                    }
-                };
-                auto fold = [&](int32_t key, float w, unsigned &grp) -> float {
-                    grp = __match_any_sync(0xFFFFFFFFu, key);
-                    if (W) {
-                        // all weights of the batch equal (e.g. the paper's default
-                        // weight 1): the group total is count * w, the correctly
-                        // rounded sum (exact for integer-valued weights)
-                        const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
-                        if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
-                        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-                        return maxn > 1 ? group_sum(grp, w, maxn) : w;
-                    }
-                    return (float)__popc(grp);
-                };
-                const uint32_t d = dk[u];
-                if (d <= 32) {
-                    // one batch: the match_any groups ARE the label totals -- no table
+                return (float)__popc(grp);
+            };
+            if (dk <= 32) {
+                // one batch: the match_any groups ARE the label totals -- no table
+                unsigned grp;
+                const float x = fold(k0, w0, grp);
+                if (k0 != kEmpty && lane == __ffs(grp) - 1) offer(x, k0);
+            } else {
+                ++tag;
+                auto batch = [&](int32_t key, float w) {
                     unsigned grp;
-                    const float x = fold(k0[u], w0[u], grp);
-                    if (k0[u] != kEmpty && lane == __ffs(grp) - 1) offer(x, k0[u]);
-                } else {
-                    ++tag;
-                    auto batch = [&](int32_t key, float w) {
-                        unsigned grp;
-                        const float x = fold(key, w, grp);
-                        if (key != kEmpty && lane == __ffs(grp) - 1) offer(tt_add<kWarpTab - 1>(tk, tv, tag, key, x), key);
-                        __syncwarp();
-                    };
-                    batch(k0[u], w0[u]);
-                    batch(k1[u], w1[u]);
-                    for (uint32_t b = 64; b < d; b += 64) {
-                        const bool u0 = b + lane < d, u1 = b + 32 + lane < d;
-                        const int32_t i0 = u0 ? __ldcs(a.indices + ok[u] + b + lane) : -1;
-                        const int32_t i1 = u1 ? __ldcs(a.indices + ok[u] + b + 32 + lane) : -1;
-                        float x0 = 0.0f, x1 = 0.0f;
-                        if (W) {
-                            if (u0) x0 = __ldcs(a.weights + ok[u] + b + lane);
-                            if (u1) x1 = __ldcs(a.weights + ok[u] + b + 32 + lane);
-                        }
-                        const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk[u]) ? a.lab_in[i0] : kEmpty;
-                        const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk[u]) ? a.lab_in[i1] : kEmpty;
-                        batch(q0, x0);
-                        if (b + 32 < d) batch(q1, x1);
+                    const float x = fold(key, w, grp);
+                    if (key != kEmpty && lane == __ffs(grp) - 1) offer(tt_add<kWarpTab - 1>(tk, tv, tag, key, x), key);
+                    __syncwarp();
+                };
+                batch(k0, w0);
+                batch(k1, w1);
+                for (uint32_t b = 64; b < dk; b += 64) {
+                    const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
+                    const int32_t i0 = u0 ? __ldcs(a.indices + ok + b + lane) : -1;
+                    const int32_t i1 = u1 ? __ldcs(a.indices + ok + b + 32 + lane) : -1;
+                    float x0 = 0.0f, x1 = 0.0f;
+                    if (W) {
+                        if (u0) x0 = __ldcs(a.weights + ok + b + lane);
+                        if (u1) x1 = __ldcs(a.weights + ok + b + 32 + lane);
                     }
+                    const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
+                    const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
+                    batch(q0, x0);
+                    if (b + 32 < dk) batch(q1, x1);
                 }
-                // hashtableMaxKey: max weight, then first label in tie order
-                const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
-                int32_t cs = kEmpty;
-                if (W1) {
-                    const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
-                    cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
-                }
-                const bool changed = accept_move(cs, cik[u], a.pickless);
-                if (changed) {
-                    if (lane == 0) a.lab_out[vk[u]] = cs;
-                    if (j0[u] >= 0) a.flag_out[j0[u]] = 1;  // mark neighbours unprocessed
-                    if (j1[u] >= 0) a.flag_out[j1[u]] = 1;
-                    for (uint32_t b = 64 + lane; b < d; b += 32) a.flag_out[a.indices[ok[u] + b]] = 1;
-                }
-                c_act += 1;
-                c_edges += d;
-                c_ch += changed;
-                c_che += changed ? d : 0;
             }
+            // hashtableMaxKey: max weight, then first label in tie order
+            const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
+            int32_t cs = kEmpty;
+            if (W1) {
+                const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
+                cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
+            }
+            const bool changed = accept_move(cs, cik, a.pickless);
+            if (changed) {
+                if (lane == 0) a.lab_out[vk] = cs;
+                if (j0 >= 0) a.flag_out[j0] = 1;            // mark neighbours unprocessed
+                if (j1 >= 0) a.flag_out[j1] = 1;
+                for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[a.indices[ok + b]] = 1;
+            }
+            c_act += 1;
+            c_edges += dk;
+            c_ch += changed;
+            c_che += changed ? dk : 0;
         }
     }
     if (lane == 0 && c_act) {
@@ -860,6 +814,7 @@ struct GiantArgs {
     int32_t *occ_n;              // [ng]
     uint8_t *active;             // [ng]
     uint8_t *changed;            // [ng]
+    unsigned long long *best;    // [ng] packed (weight, tie rank) maximum
 };
 
 template <bool SYNC>
@@ -870,6 +825,7 @@ __global__ void k_giant_snapshot(SweepArgs a, GiantArgs g, int64_t ng) {
     uint8_t f = a.flag_in[v];
     g.active[k] = f ? 1 : 0;
     g.changed[k] = 0;
+    g.best[k] = 0;
     if (!SYNC && f) a.flag_in[v] = 0;
 }
 
@@ -920,28 +876,34 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
     if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
 }
 
+// hashtableMaxKey for giant vertices, spread over the vertex's chunk CTAs:
+// CTA k of a vertex scans occupied-list entries [k*kGiantChunk, ...), clears
+// those slots, and folds its maximum into best[gi] (global 64-bit atomicMax).
 template <bool SYNC, int TIE>
-__global__ void __launch_bounds__(kBlockThreads) k_giant_finalize(SweepArgs a, GiantArgs g) {
-    const int64_t gi = blockIdx.x;
+__global__ void __launch_bounds__(kBlockThreads) k_giant_reduce(SweepArgs a, GiantArgs g) {
+    const int64_t c = blockIdx.x;
+    const int32_t gi = g.chunk_g[c];
     if (!g.active[gi]) return;
     __shared__ uint64_t red[kBlockThreads / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int32_t r = g.verts[gi];
+    const int64_t kc = (g.chunk_e0[c] - a.offsets[r]) / kGiantChunk;
     int32_t *gk = g.keys + g.table_off[gi];
     float *gv = g.vals + g.table_off[gi];
     const int32_t *occ = g.occ + g.table_off[gi];
-    const int32_t cnt = g.occ_n[gi];
-    const int32_t r = g.verts[gi];
+    const int64_t cnt = g.occ_n[gi];
+    const int64_t q0 = kc * kGiantChunk, q1 = q0 + kGiantChunk < cnt ? q0 + kGiantChunk : cnt;
     Hash h;
     h.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
     TieOrder<TIE> to;
     to.init(h);
     uint64_t best = 0;
-    for (int32_t q = threadIdx.x; q < cnt; q += kBlockThreads) {
-        int32_t s = occ[q];
-        uint64_t c = pack_cand(gv[s], gk[s], to);
-        best = c > best ? c : best;
-        gk[s] = kEmpty;
-        gv[s] = 0.0f;
+    for (int64_t q = q0 + threadIdx.x; q < q1; q += kBlockThreads) {
+        const int32_t sl = occ[q];
+        const uint64_t cd = pack_cand(gv[sl], gk[sl], to);
+        best = cd > best ? cd : best;
+        gk[sl] = kEmpty;
+        gv[sl] = 0.0f;
     }
     best = warp_max_u64(best);
     if (lane == 0) red[wid] = best;
@@ -949,22 +911,34 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_finalize(SweepArgs a, G
     if (wid == 0) {
         uint64_t b = lane < kBlockThreads / 32 ? red[lane] : 0;
         b = warp_max_u64(b);
-        if (lane == 0) {
-            g.occ_n[gi] = 0;
-            int64_t v = g.verts[gi] + a.row_begin;
-            int32_t ci = a.lab_in[v];
-            int32_t cs = b ? cand_label(b, to) : kEmpty;
-            bool ch = accept_move(cs, ci, a.pickless);
-            if (ch) {
-                a.lab_out[v] = cs;
-                g.changed[gi] = 1;
-                atomicAdd(&a.ctr[0], 1ull);
-                atomicAdd(&a.ctr[9 + 3], 1ull);
-                atomicAdd(&a.ctr[13 + 3], (unsigned long long)(a.offsets[r + 1] - a.offsets[r]));
-            }
-            atomicAdd(&a.ctr[1 + 3], 1ull);
-        }
+        if (lane == 0 && b) atomicMax(&g.best[gi], (unsigned long long)b);
     }
+}
+
+// the move rule for every giant vertex (one thread each)
+template <bool SYNC, int TIE>
+__global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
+    const int64_t gi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (gi >= ng || !g.active[gi]) return;
+    g.occ_n[gi] = 0;
+    const int32_t r = g.verts[gi];
+    const int64_t v = r + a.row_begin;
+    const int64_t deg = a.offsets[r + 1] - a.offsets[r];
+    Hash h;
+    h.init((uint32_t)deg);
+    TieOrder<TIE> to;
+    to.init(h);
+    const unsigned long long b = g.best[gi];
+    const int32_t cs = b ? cand_label(b, to) : kEmpty;
+    const bool ch = accept_move(cs, a.lab_in[v], a.pickless);
+    if (ch) {
+        a.lab_out[v] = cs;
+        g.changed[gi] = 1;
+        atomicAdd(&a.ctr[0], 1ull);
+        atomicAdd(&a.ctr[9 + 3], 1ull);
+        atomicAdd(&a.ctr[13 + 3], (unsigned long long)deg);
+    }
+    atomicAdd(&a.ctr[1 + 3], 1ull);
 }
 
 __global__ void __launch_bounds__(kBlockThreads) k_giant_mark(SweepArgs a, GiantArgs g) {
@@ -1219,6 +1193,7 @@ struct nulpa_graph {
     int32_t *gkeys = nullptr, *occ = nullptr, *occ_n = nullptr;
     float *gvals = nullptr;
     uint8_t *gactive = nullptr, *gchanged = nullptr;
+    unsigned long long *gbest = nullptr;
     // counters
     unsigned long long *ctr = nullptr;       // device [kMaxIter+1][kCtr]
     unsigned long long *ctr_host = nullptr;  // pinned
@@ -1262,6 +1237,8 @@ void free_bins(nulpa_graph *g) {
     cudaFree(g->occ_n);
     cudaFree(g->gactive);
     cudaFree(g->gchanged);
+    cudaFree(g->gbest);
+    g->gbest = nullptr;
     g->chunk_g = nullptr;
     g->chunk_e0 = g->chunk_e1 = g->table_off = nullptr;
     g->gkeys = g->occ = g->occ_n = nullptr;
@@ -1359,6 +1336,7 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CHECK(dalloc(&g->occ_n, (size_t)ng));
         CHECK(dalloc(&g->gactive, (size_t)ng));
         CHECK(dalloc(&g->gchanged, (size_t)ng));
+        CHECK(dalloc(&g->gbest, (size_t)ng));
         CU(cudaMemcpy(g->chunk_g, cg.data(), cg.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
         CU(cudaMemcpy(g->chunk_e0, c0.data(), c0.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
         CU(cudaMemcpy(g->chunk_e1, c1.data(), c1.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
@@ -1460,6 +1438,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             ga.occ_n = g->occ_n;
             ga.active = g->gactive;
             ga.changed = g->gchanged;
+            ga.best = g->gbest;
             const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float));
             static bool attr_set = false;   // one per template instantiation
             if (!attr_set) {
@@ -1468,10 +1447,11 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             }
             k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, g->stream>>>(a, ga, ng);
             k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, g->stream>>>(a, ga);
-            k_giant_finalize<SYNC, TIE><<<(unsigned)ng, kBlockThreads, 0, g->stream>>>(a, ga);
+            k_giant_reduce<SYNC, TIE><<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
+            k_giant_decide<SYNC, TIE><<<grid_for(ng, 128), 128, 0, g->stream>>>(a, ga, ng);
             k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
             CU(cudaGetLastError());
-            g->stats.launches[3] += 4;
+            g->stats.launches[3] += 5;
         }
         CHECK(rec(3, 1));
         return NULPA_OK;
@@ -1492,12 +1472,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[1];
         CHECK(rec(1, 0));
         if (n > 0) {
-            static bool attr_set = false;
-            if (!attr_set) {
-                CU(cudaFuncSetAttribute(k_warp<SYNC, W, TIE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sizeof(WarpSmem) * (kWarpThreads / 32))));
-                attr_set = true;
-            }
-            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * 4), kWarpThreads, sizeof(WarpSmem) * (kWarpThreads / 32), g->stream>>>(a, g->bin_list[1], n);
+            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * kWarpCtasPerSm), kWarpThreads, 0, g->stream>>>(a, g->bin_list[1], n);
             CU(cudaGetLastError());
             g->stats.launches[1] += 1;
         }
