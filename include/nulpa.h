@@ -69,7 +69,9 @@ typedef struct nulpa_params {
                                     home slot k mod p1, then smallest label (PAPER.md:173
                                     "selects the first label with the highest associated weight") */
     int32_t bin_order;           /* 1 (default): thread, warp, block, giant bins in that order
-                                    within a sweep (hubs last); 0: giant, block, warp, thread    */
+                                    within a sweep (hubs last); 0: giant, block, warp, thread;
+                                    2: block + giant on a second stream, concurrent with
+                                    thread + warp                                               */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0

@@ -1205,6 +1205,8 @@ struct nulpa_graph {
     cudaEvent_t ev[2 * 4 * (kMaxIter + 1)];
     cudaEvent_t ev_run[2];
     bool events = false;
+    cudaStream_t side = nullptr;             // bin_order 2: block + giant bins
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     nulpa_stats stats;
 };
 
@@ -1367,7 +1369,7 @@ int validate_params(const nulpa_params &p) {
     if (p.block_degree < p.switch_degree || p.block_degree > 256)
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
-    if (p.bin_order != 0 && p.bin_order != 1) return fail(NULPA_EINVAL, "bin_order must be 0 or 1");
+    if (p.bin_order < 0 || p.bin_order > 2) return fail(NULPA_EINVAL, "bin_order must be 0, 1 or 2");
     if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
         return fail(NULPA_EINVAL, "giant_degree must be in [block_degree, 4096] (CTA tables hold 4095 slots)");
     return NULPA_OK;
@@ -1418,8 +1420,9 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     a.lab_out = g->labels;
     a.flag_out = g->flags;
     const int sms = num_sms();
+    cudaStream_t cs = g->stream;                  // stream of the bin being launched
     auto rec = [&](int b, int which) -> int {
-        if (timing) CU(cudaEventRecord(g->ev[(slot * 4 + b) * 2 + which], g->stream));
+        if (timing) CU(cudaEventRecord(g->ev[(slot * 4 + b) * 2 + which], cs));
         return NULPA_OK;
     };
     auto run_giant = [&]() -> int {
@@ -1445,11 +1448,11 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                 CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
                 attr_set = true;
             }
-            k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, g->stream>>>(a, ga, ng);
-            k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, g->stream>>>(a, ga);
-            k_giant_reduce<SYNC, TIE><<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
-            k_giant_decide<SYNC, TIE><<<grid_for(ng, 128), 128, 0, g->stream>>>(a, ga, ng);
-            k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, g->stream>>>(a, ga);
+            k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, cs>>>(a, ga, ng);
+            k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
+            k_giant_reduce<SYNC, TIE><<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
+            k_giant_decide<SYNC, TIE><<<grid_for(ng, 128), 128, 0, cs>>>(a, ga, ng);
+            k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
             CU(cudaGetLastError());
             g->stats.launches[3] += 5;
         }
@@ -1461,7 +1464,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(2, 0));
         if (n > 0) {
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, g->stream>>>(a, g->bin_list[2], n);
+            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, g->bin_list[2], n);
             CU(cudaGetLastError());
             g->stats.launches[2] += 1;
         }
@@ -1472,7 +1475,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[1];
         CHECK(rec(1, 0));
         if (n > 0) {
-            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * kWarpCtasPerSm), kWarpThreads, 0, g->stream>>>(a, g->bin_list[1], n);
+            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * kWarpCtasPerSm), kWarpThreads, 0, cs>>>(a, g->bin_list[1], n);
             CU(cudaGetLastError());
             g->stats.launches[1] += 1;
         }
@@ -1494,6 +1497,24 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(run_block());
         CHECK(run_warp());
         CHECK(run_thread());
+    } else if (p.bin_order == 2) {
+        // block + giant bins on a side stream, concurrent with thread + warp:
+        // their latency-bound CTAs fill the SMs the warp bin leaves idle
+        if (!g->side) {
+            CU(cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking));
+            CU(cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming));
+            CU(cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming));
+        }
+        CU(cudaEventRecord(g->ev_fork, g->stream));
+        CU(cudaStreamWaitEvent(g->side, g->ev_fork, 0));
+        cs = g->side;
+        CHECK(run_block());
+        CHECK(run_giant());
+        CU(cudaEventRecord(g->ev_join, g->side));
+        cs = g->stream;
+        CHECK(run_thread());
+        CHECK(run_warp());
+        CU(cudaStreamWaitEvent(g->stream, g->ev_join, 0));
     } else {
         CHECK(run_thread());
         CHECK(run_warp());
@@ -1858,6 +1879,12 @@ int nulpa_destroy(nulpa_graph *g) {
     if (g->ctr_host) cudaFreeHost(g->ctr_host);
     cudaFree(g->Sigma);
     cudaFree(g->macc);
+    if (g->side) {
+        cudaStreamSynchronize(g->side);
+        cudaStreamDestroy(g->side);
+        cudaEventDestroy(g->ev_fork);
+        cudaEventDestroy(g->ev_join);
+    }
     if (g->events) {
         for (auto &e : g->ev) cudaEventDestroy(e);
         cudaEventDestroy(g->ev_run[0]);
