@@ -1085,48 +1085,97 @@ __global__ void k_gather_degrees(const int64_t *offsets, const int32_t *rows, in
 // ---------------------------------------------------------------------------
 // modularity (Eq. 1, second form, R11), float64
 // ---------------------------------------------------------------------------
-// acc[0] += sigma_intra, acc[1] += 2m; Sigma[c] += K_i
+// K_i = sum_j w_ij for every row (float64), computed once per handle; acc[1] += 2m
 template <bool W>
-__global__ void __launch_bounds__(256) k_mod_rows(const int64_t *__restrict__ offsets, const int32_t *__restrict__ indices,
-                                                  const float *__restrict__ weights, const int32_t *__restrict__ labels,
-                                                  int64_t n_rows, int64_t row_begin, double *Sigma, double *acc) {
+__global__ void __launch_bounds__(256) k_mod_degrees(const int64_t *__restrict__ offsets, const float *__restrict__ weights,
+                                                     int64_t n_rows, double *K, double *acc) {
     const int lane = threadIdx.x & 31;
     const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
-    double intra = 0.0, tot = 0.0;
+    double tot = 0.0;
     for (int64_t r = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); r < n_rows; r += nw) {
-        int64_t v = r + row_begin;
-        int32_t cv = labels[v];
-        double K = 0.0, in = 0.0;
-        for (int64_t e = offsets[r] + lane; e < offsets[r + 1]; e += 32) {
-            double w = W ? (double)weights[e] : 1.0;
-            K += w;
-            if (labels[indices[e]] == cv) in += w;
-        }
+        double k = 0.0;
+        if (W) {
+            for (int64_t e = offsets[r] + lane; e < offsets[r + 1]; e += 32) k += (double)weights[e];
 #pragma unroll
-        for (int o = 16; o; o >>= 1) {
-            K += __shfl_xor_sync(0xFFFFFFFFu, K, o);
-            in += __shfl_xor_sync(0xFFFFFFFFu, in, o);
+            for (int o = 16; o; o >>= 1) k += __shfl_xor_sync(0xFFFFFFFFu, k, o);
+        } else {
+            k = (double)(offsets[r + 1] - offsets[r]);
         }
         if (lane == 0) {
-            if (K != 0.0) atomicAdd(&Sigma[cv], K);
-            intra += in;
-            tot += K;
+            K[r] = k;
+            tot += k;
         }
     }
-    __shared__ double s_in[8], s_tot[8];
-    if (lane == 0) {
-        s_in[threadIdx.x >> 5] = intra;
-        s_tot[threadIdx.x >> 5] = tot;
+    if (lane == 0) atomicAdd(&acc[1], tot);
+}
+
+// acc[0] += sigma_intra = sum over CSR entries (i,j) with C_i = C_j of w_ij.
+// A warp takes 32 consecutive rows (their labels / offsets in one round
+// trip) and strides over each row's entries; per-lane float64 partial sums,
+// reduced once at the end.
+template <bool W>
+__global__ void __launch_bounds__(256) k_mod_intra(const int64_t *__restrict__ offsets, const int32_t *__restrict__ indices,
+                                                   const float *__restrict__ weights, const int32_t *__restrict__ labels,
+                                                   int64_t n_rows, int64_t row_begin, double *acc) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x / 32);
+    const int64_t nchunks = (n_rows + 31) / 32;
+    double in = 0.0;
+    for (int64_t c = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); c < nchunks; c += nw) {
+        const int64_t r = c * 32 + lane;
+        int32_t cv = 0;
+        int64_t o0 = 0, o1 = 0;
+        if (r < n_rows) {
+            cv = labels[r + row_begin];
+            o0 = offsets[r];
+            o1 = offsets[r + 1];
+        }
+        for (int k = 0; k < 32; ++k) {
+            const int32_t ck = __shfl_sync(0xFFFFFFFFu, cv, k);
+            const int64_t b = __shfl_sync(0xFFFFFFFFu, o0, k), e1 = __shfl_sync(0xFFFFFFFFu, o1, k);
+            for (int64_t e = b + lane; e < e1; e += 32)
+                if (labels[__ldcs(indices + e)] == ck) in += W ? (double)__ldcs(weights + e) : 1.0;
+        }
     }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) in += __shfl_xor_sync(0xFFFFFFFFu, in, o);
+    __shared__ double s_in[8];
+    if (lane == 0) s_in[threadIdx.x >> 5] = in;
     __syncthreads();
     if (threadIdx.x == 0) {
-        double a = 0, b = 0;
-        for (int w = 0; w < (int)(blockDim.x / 32); ++w) {
-            a += s_in[w];
-            b += s_tot[w];
-        }
-        atomicAdd(&acc[0], a);
-        atomicAdd(&acc[1], b);
+        double t = 0;
+        for (int w = 0; w < (int)(blockDim.x / 32); ++w) t += s_in[w];
+        atomicAdd(&acc[0], t);
+    }
+}
+
+// Sigma[C_i] += K_i, one thread per row; rows of a warp holding the same
+// label are summed first (match_any + pairwise tree) so a community costs
+// one atomicAdd per warp instead of one per vertex.
+__device__ __forceinline__ double group_sum_d(unsigned grp, double x, unsigned maxn) {
+    const int lane = threadIdx.x & 31;
+    const unsigned rank = __popc(grp & ((1u << lane) - 1));
+    const unsigned above = lane == 31 ? 0u : grp & (0xFFFFFFFEu << lane);
+    int nxt = above ? __ffs(above) - 1 : 32;
+    for (unsigned d = 1; d < maxn; d <<= 1) {
+        const double y = __shfl_sync(0xFFFFFFFFu, x, nxt & 31);
+        const int n2 = __shfl_sync(0xFFFFFFFFu, nxt, nxt & 31);
+        if ((rank & (2 * d - 1)) == 0 && nxt < 32) x += y;
+        nxt = nxt < 32 ? n2 : 32;
+    }
+    return x;
+}
+__global__ void __launch_bounds__(256) k_mod_sigma(const double *__restrict__ K, const int32_t *__restrict__ labels,
+                                                   int64_t n_rows, int64_t row_begin, double *Sigma) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n_rows; base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = base + threadIdx.x;
+        const int32_t c = r < n_rows ? labels[r + row_begin] : -1;
+        const double k = r < n_rows ? K[r] : 0.0;
+        const unsigned grp = __match_any_sync(0xFFFFFFFFu, c);
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, (unsigned)__popc(grp));
+        const double s = maxn > 1 ? group_sum_d(grp, k, maxn) : k;
+        if (c >= 0 && lane == __ffs(grp) - 1 && s != 0.0) atomicAdd(&Sigma[c], s);
     }
 }
 
@@ -1201,6 +1250,8 @@ struct nulpa_graph {
     // modularity scratch
     double *Sigma = nullptr;
     double *macc = nullptr;
+    double *Kdeg = nullptr;                  // K_i (float64), cached by the first modularity call
+    double two_m_local = 0.0;
     // timing
     cudaEvent_t ev[2 * 4 * (kMaxIter + 1)];
     cudaEvent_t ev_run[2];
@@ -1797,17 +1848,31 @@ int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, doubl
     if (!g->macc) CHECK(dalloc(&g->macc, 4));
     const int32_t *lab = labels_device ? labels_device : g->labels;
     CU(cudaMemsetAsync(g->macc, 0, 4 * sizeof(double), g->stream));
-    const int grid = grid_for(g->n_rows, 8, num_sms() * 8);
+    const int sms = num_sms();
+    if (!g->Kdeg) {                                         // graph-invariant: K_i and 2m, once
+        CHECK(dalloc(&g->Kdeg, (size_t)std::max<int64_t>(g->n_rows, 1)));
+        if (g->weights)
+            k_mod_degrees<true><<<sms * 8, 256, 0, g->stream>>>(g->offsets, g->weights, g->n_rows, g->Kdeg, g->macc);
+        else
+            k_mod_degrees<false><<<sms * 8, 256, 0, g->stream>>>(g->offsets, g->weights, g->n_rows, g->Kdeg, g->macc);
+        CU(cudaGetLastError());
+        double h2[4];
+        CU(cudaMemcpyAsync(h2, g->macc, sizeof h2, cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        g->two_m_local = h2[1];
+        CU(cudaMemsetAsync(g->macc, 0, 4 * sizeof(double), g->stream));
+    }
     if (g->weights)
-        k_mod_rows<true><<<grid, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, Sigma_device, g->macc);
+        k_mod_intra<true><<<sms * 8, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, g->macc);
     else
-        k_mod_rows<false><<<grid, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, Sigma_device, g->macc);
+        k_mod_intra<false><<<sms * 8, 256, 0, g->stream>>>(g->offsets, g->indices, g->weights, lab, g->n_rows, g->row_begin, g->macc);
+    k_mod_sigma<<<sms * 8, 256, 0, g->stream>>>(g->Kdeg, lab, g->n_rows, g->row_begin, Sigma_device);
     CU(cudaGetLastError());
     double h[4];
     CU(cudaMemcpyAsync(h, g->macc, sizeof h, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
     *sigma_intra += h[0];
-    *two_m += h[1];
+    *two_m += g->two_m_local;
     return NULPA_OK;
 }
 
@@ -1879,6 +1944,7 @@ int nulpa_destroy(nulpa_graph *g) {
     if (g->ctr_host) cudaFreeHost(g->ctr_host);
     cudaFree(g->Sigma);
     cudaFree(g->macc);
+    cudaFree(g->Kdeg);
     if (g->side) {
         cudaStreamSynchronize(g->side);
         cudaStreamDestroy(g->side);
