@@ -304,37 +304,13 @@ __device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, i
     }
 }
 
-// One 32-edge batch of a warp against the warp's PRIVATE table: lanes
-// holding the same label (match_any) are folded onto their lowest lane (the
-// leader), which claims the label's slot (Algorithm 2 probing, atomicCAS on
-// the key) and adds the group's weight with a plain shared-memory
-// read-modify-write -- no other lane of the batch touches that slot, and
-// batches are ordered by __syncwarp, so no float atomics are needed (the GPU
-// has no native shared-memory float atomicAdd).  Unit weights: the group
-// weight is the member count, exact.  key == kEmpty marks an idle lane.
-template <bool W>
-__device__ __forceinline__ void warp_batch_accumulate(int32_t *Hk, float *Hv, const Hash &h, int32_t key, float w) {
-    const int lane = threadIdx.x & 31;
-    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
-    const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
-    float sum;
-    if (W) {
-        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
-    } else {
-        sum = (float)__popc(grp);
-    }
-    if (leader) {
-        const uint32_t slot = ht_claim(Hk, h, key);
-        Hv[slot] = __fadd_rn(Hv[slot], sum);
-    }
-    __syncwarp();
-}
-
-// The same folding for a table shared by several warps (block / giant
-// kernels): the leader adds its group's sum with one shared-memory
-// atomicAdd (a CAS loop on this GPU, now contended by at most one lane per
-// warp and label).
+// One 32-edge batch of a warp against a table shared by several warps (the
+// giant chunk tables): lanes holding the same label (match_any) are folded
+// onto their lowest lane (the leader), which claims the label's slot
+// (Algorithm 2 probing, atomicCAS) and adds the group's total with one
+// shared-memory atomicAdd (a CAS loop on this GPU -- there is no native
+// shared float atomicAdd -- contended by at most one lane per warp and
+// label).  Uniform weights: total = count * w.
 template <bool W>
 __device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float *Hv, const Hash &h, int32_t key,
                                                              float w) {
@@ -343,8 +319,14 @@ __device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float 
     const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
     float sum;
     if (W) {
-        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-        sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
+        const unsigned valid = __ballot_sync(0xFFFFFFFFu, key != kEmpty);
+        const float wr = __shfl_sync(0xFFFFFFFFu, w, valid ? __ffs(valid) - 1 : 0);
+        if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == wr)) {
+            sum = (float)__popc(grp) * w;
+        } else {
+            const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+            sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
+        }
     } else {
         sum = (float)__popc(grp);
     }
