@@ -370,6 +370,7 @@ def run_distributed(args, rank, world, local):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
     dist.barrier()
+    st_a = runner.g.stats()
     ev0.record()
     res = None
     for _ in range(args.steps):
@@ -378,6 +379,8 @@ def run_distributed(args, rank, world, local):
     torch.cuda.synchronize()
     dist.barrier()
     ck = clocks.stop()
+    st_b = runner.g.stats()
+    launches = (sum(st_b["launches"]) + st_b["other_launches"]) - (sum(st_a["launches"]) + st_a["other_launches"])
     ms = torch.tensor([ev0.elapsed_time(ev1) / args.steps], dtype=torch.float64, device="cuda")
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms = float(ms.item())
@@ -389,7 +392,7 @@ def run_distributed(args, rank, world, local):
                 "config": {"workload": args.config, "N": shard.N_global, "M": shard.M_global, "weights": args.weights,
                            "parallelism": f"vertex range split by edge count over {world} GPUs, NCCL all-gather of labels per sweep"},
                 "iterations": res["iterations"], "changed": res["changed"], "modularity": q,
-                "gpu_launches": res["launches"] * args.steps, "clocks": ck}
+                "gpu_launches": launches, "clocks": ck}
         print(json.dumps(line), flush=True)
     dist.barrier()
     dist.destroy_process_group()
