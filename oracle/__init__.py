@@ -67,12 +67,31 @@ def _L():
         lib.oracle_lpa.restype = ctypes.c_int
         lib.oracle_modularity.argtypes = [i64, vp, vp, vp, vp]
         lib.oracle_modularity.restype = f64
+        lib.oracle_set_tie_rule.argtypes = [ctypes.c_int]
+        lib.oracle_set_tie_rule.restype = None
         _lib = lib
     return _lib
 
 
 def _p(a):
     return None if a is None else a.ctypes.data
+
+
+TIE_SMALLEST, TIE_SLOT = 0, 1
+
+
+class _tie:
+    """Select the tie order of hashtableMaxKey for one call (R6): 0 smallest
+    label (north star), 1 smallest home slot k mod p1 then smallest label."""
+
+    def __init__(self, rule):
+        self.rule = int(rule)
+
+    def __enter__(self):
+        _L().oracle_set_tie_rule(self.rule)
+
+    def __exit__(self, *exc):
+        _L().oracle_set_tie_rule(0)
 
 
 class CSR:
@@ -129,36 +148,39 @@ class Hashtable:
                                                   int(k), float(v), max_retries, ctypes.byref(slot))
         return probes, slot.value
 
-    def max_key(self):
+    def max_key(self, tie_rule: int = 0):
         w1, w2 = ctypes.c_float(), ctypes.c_float()
-        k = _L().oracle_hashtable_max_key(_p(self.Hk), _p(self.Hv), self.p1, ctypes.byref(w1), ctypes.byref(w2))
+        with _tie(tie_rule):
+            k = _L().oracle_hashtable_max_key(_p(self.Hk), _p(self.Hv), self.p1, ctypes.byref(w1), ctypes.byref(w2))
         return k, w1.value, w2.value
 
 
 # --- Algorithm 1 ------------------------------------------------------------------
 
-def vertex_best(g, i: int, labels):
+def vertex_best(g, i: int, labels, tie_rule: int = 0):
     g = as_csr(g)
     labels = np.ascontiguousarray(labels, dtype=np.int32)
     w1, w2 = ctypes.c_float(), ctypes.c_float()
-    c = _L().oracle_vertex_best(int(i), _p(g.offsets), _p(g.indices), _p(g.weights), _p(labels),
-                                ctypes.byref(w1), ctypes.byref(w2))
+    with _tie(tie_rule):
+        c = _L().oracle_vertex_best(int(i), _p(g.offsets), _p(g.indices), _p(g.weights), _p(labels),
+                                    ctypes.byref(w1), ctypes.byref(w2))
     return int(c), w1.value, w2.value
 
 
-def lpa_move_async(g, labels, unprocessed, pickless: bool):
+def lpa_move_async(g, labels, unprocessed, pickless: bool, tie_rule: int = 0):
     """One asynchronous lpaMove; updates labels / unprocessed IN PLACE; returns Delta N."""
     g = as_csr(g)
     assert labels.dtype == np.int32 and labels.flags.c_contiguous
     assert unprocessed.dtype == np.uint8 and unprocessed.flags.c_contiguous
     buf_k = np.empty(2 * g.M + 1, dtype=np.int32)
     buf_v = np.empty(2 * g.M + 1, dtype=np.float32)
-    return int(_L().oracle_lpa_move_async(g.N, _p(g.offsets), _p(g.indices), _p(g.weights),
-                                          _p(labels), _p(unprocessed), int(bool(pickless)),
-                                          _p(buf_k), _p(buf_v)))
+    with _tie(tie_rule):
+        return int(_L().oracle_lpa_move_async(g.N, _p(g.offsets), _p(g.indices), _p(g.weights),
+                                              _p(labels), _p(unprocessed), int(bool(pickless)),
+                                              _p(buf_k), _p(buf_v)))
 
 
-def lpa_move_sync(g, labels, unprocessed, pickless: bool):
+def lpa_move_sync(g, labels, unprocessed, pickless: bool, tie_rule: int = 0):
     """One synchronous (Jacobi) lpaMove.  Returns (dN, new_labels, new_unprocessed, w1, w2)."""
     g = as_csr(g)
     C_old = np.ascontiguousarray(labels, dtype=np.int32)
@@ -169,20 +191,23 @@ def lpa_move_sync(g, labels, unprocessed, pickless: bool):
     w2 = np.empty(g.N, dtype=np.float32)
     buf_k = np.empty(2 * g.M + 1, dtype=np.int32)
     buf_v = np.empty(2 * g.M + 1, dtype=np.float32)
-    dN = _L().oracle_lpa_move_sync(g.N, _p(g.offsets), _p(g.indices), _p(g.weights), _p(C_old), _p(C_new),
-                                   _p(U_old), _p(U_new), int(bool(pickless)), _p(buf_k), _p(buf_v),
-                                   _p(w1), _p(w2))
+    with _tie(tie_rule):
+        dN = _L().oracle_lpa_move_sync(g.N, _p(g.offsets), _p(g.indices), _p(g.weights), _p(C_old), _p(C_new),
+                                       _p(U_old), _p(U_new), int(bool(pickless)), _p(buf_k), _p(buf_v),
+                                       _p(w1), _p(w2))
     return int(dN), C_new, U_new, w1, w2
 
 
-def lpa(g, tolerance: float = 0.05, max_iterations: int = 20, pickless_period: int = 4, sync: bool = False):
+def lpa(g, tolerance: float = 0.05, max_iterations: int = 20, pickless_period: int = 4, sync: bool = False,
+        tie_rule: int = 0):
     """Algorithm 1 lpa().  Returns (labels, iterations, dN_per_iteration).
     Defaults are the paper's: tau = 0.05, 20 iterations, PL every 4."""
     g = as_csr(g)
     C = np.empty(g.N, dtype=np.int32)
     dN = np.zeros(max(max_iterations, 1), dtype=np.int64)
-    it = _L().oracle_lpa(g.N, _p(g.offsets), _p(g.indices), _p(g.weights), _p(C), float(tolerance),
-                         int(max_iterations), int(pickless_period), int(bool(sync)), _p(dN))
+    with _tie(tie_rule):
+        it = _L().oracle_lpa(g.N, _p(g.offsets), _p(g.indices), _p(g.weights), _p(C), float(tolerance),
+                             int(max_iterations), int(pickless_period), int(bool(sync)), _p(dN))
     return C, int(it), dN[:it].copy()
 
 

@@ -32,11 +32,19 @@ def adjacency(g):
             for i in range(g.N)]
 
 
-def naive_best(i, adj_i, C):
+def naive_best(i, adj_i, C, tie_rule=0):
     """Brute force Eq. 3: enumerate candidate labels in
-    increasing order, sum float32 weights in CSR order, keep the strictly
-    larger -> max weight, smallest label on ties (R6)."""
+    tie order (R6: increasing label; tie rule 1: increasing home slot
+    c mod p1 with p1 = nextPow2(D)-1, then label), sum float32 weights in CSR
+    order, keep the strictly larger."""
     cands = sorted({C[j] for j, _ in adj_i if j != i})
+    if tie_rule == 1:
+        D = len(adj_i)
+        p1 = 1
+        while p1 <= D:
+            p1 *= 2
+        p1 -= 1
+        cands = sorted(cands, key=lambda c: ((c % p1), c))
     best, bw, all_w = None, None, []
     for c in cands:
         s = np.float32(0.0)
@@ -156,16 +164,17 @@ def test_hashtable_tie_takes_smallest_label():
 # one vertex / one sweep against brute force
 # ---------------------------------------------------------------------------
 
+@pytest.mark.parametrize("tie_rule", [0, 1])
 @pytest.mark.parametrize("weighted", [False, True])
 @pytest.mark.parametrize("seed", [0, 1, 2])
-def test_vertex_best_bruteforce(weighted, seed):
+def test_vertex_best_bruteforce(weighted, seed, tie_rule):
     g = np_graph(synth.erdos_renyi(60, 400, seed=seed, weighted=weighted))
     rng = np.random.default_rng(seed)
-    C = rng.integers(0, 12, g.N).astype(np.int32)   # few labels -> many collisions/ties
+    C = rng.integers(0, 40, g.N).astype(np.int32)   # few labels -> many collisions/ties
     adj = adjacency(g)
     for i in range(g.N):
-        c, w1, w2 = oracle.vertex_best(g, i, C)
-        nc, nw1, nw2 = naive_best(i, adj[i], C)
+        c, w1, w2 = oracle.vertex_best(g, i, C, tie_rule=tie_rule)
+        nc, nw1, nw2 = naive_best(i, adj[i], C, tie_rule)
         if nc is None:
             assert c == oracle.EMPTY
             continue
