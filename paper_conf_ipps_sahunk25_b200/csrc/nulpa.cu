@@ -269,30 +269,44 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
 // distinct (one leader per label), batches are ordered by __syncwarp, so the
 // value update is a plain read-modify-write; only the slot claim is atomic
 // (64-bit shared-memory CAS).
+__device__ __forceinline__ uint64_t lds_u64(uint32_t addr) {
+    uint64_t v;
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ float lds_f32(uint32_t addr) {
+    float v;
+    asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
+    asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t cas_u64(uint32_t addr, uint64_t cmp, uint64_t val) {
+    uint64_t old;
+    asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(addr), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+
+// Full probe sequence (collisions, lost claim races): out of line.
 template <uint32_t P1>
-__device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, int32_t k, float x) {
+__device__ __noinline__ float tt_add_slow(uint32_t tk, uint32_t tv, uint32_t tag, int32_t k, float x) {
     constexpr uint32_t p1 = P1, p2 = 2 * P1 + 1;
     const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
-    uint32_t i = (uint32_t)k % p1;
-    uint32_t di = 1;
-    uint32_t km = 0xFFFFFFFFu;                             // k mod p2, computed on the first collision
+    uint32_t i = (uint32_t)k % p1, di = 1;
+    const uint32_t km = ((uint32_t)k % p2) % p1;           // 2nd hash
     for (int t = 0;; ++t) {
-        const uint64_t cur = *((volatile uint64_t *)&tk[i]);
+        const uint64_t cur = lds_u64(tk + 8 * i);
         if (cur == want) {
-            const float V = __fadd_rn(tv[i], x);
-            tv[i] = V;
+            const float V = __fadd_rn(lds_f32(tv + 4 * i), x);
+            sts_f32(tv + 4 * i, V);
             return V;
         }
-        if ((uint32_t)(cur >> 32) != tag) {                 // empty slot: claim it
-            const unsigned long long old =
-                atomicCAS((unsigned long long *)&tk[i], (unsigned long long)cur, (unsigned long long)want);
-            if (old == cur) {
-                tv[i] = x;
-                return x;
-            }
+        if ((uint32_t)(cur >> 32) != tag && cas_u64(tk + 8 * i, cur, want) == cur) {   // empty: claim
+            sts_f32(tv + 4 * i, x);
+            return x;
         }
         if (t < kMaxRetries) {
-            if (km == 0xFFFFFFFFu) km = ((uint32_t)k % p2) % p1;
             i += di;
             if (i >= p1) i -= p1;
             di = 2 * di + km;
@@ -302,6 +316,26 @@ __device__ __forceinline__ float tt_add(uint64_t *tk, float *tv, uint32_t tag, i
             i = i + 1 == p1 ? 0 : i + 1;                   // R5
         }
     }
+}
+
+// Algorithm 2's accumulate into a warp-private tagged table at shared
+// addresses tk (keys, 8 B/slot) / tv (values, 4 B/slot).  Fast path: the
+// home slot k mod p1 holds (tag, k) or is free (stale tag) and is claimed.
+template <uint32_t P1>
+__device__ __forceinline__ float tt_add(uint32_t tk, uint32_t tv, uint32_t tag, int32_t k, float x) {
+    const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
+    const uint32_t i = (uint32_t)k % P1;
+    const uint64_t cur = lds_u64(tk + 8 * i);
+    if (cur == want) {
+        const float V = __fadd_rn(lds_f32(tv + 4 * i), x);
+        sts_f32(tv + 4 * i, V);
+        return V;
+    }
+    if ((uint32_t)(cur >> 32) != tag && cas_u64(tk + 8 * i, cur, want) == cur) {
+        sts_f32(tv + 4 * i, x);
+        return x;
+    }
+    return tt_add_slow<P1>(tk, tv, tag, k, x);
 }
 
 // One 32-edge batch of a warp against a table shared by several warps (the
@@ -481,9 +515,9 @@ __global__ void __launch_bounds__(kWarpThreads, kWarpCtasPerSm) k_warp(SweepArgs
     __shared__ float s_tv[kWarpThreads / 32][kWarpTab];
     __shared__ unsigned long long bctr[4];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    uint64_t *tk = s_tk[wid];
-    float *tv = s_tv[wid];
-    for (int q = lane; q < kWarpTab; q += 32) tk[q] = 0;   // tag 0: empty for every vertex
+    const uint32_t tk = (uint32_t)__cvta_generic_to_shared(&s_tk[wid][0]);
+    const uint32_t tv = (uint32_t)__cvta_generic_to_shared(&s_tv[wid][0]);
+    for (int q = lane; q < kWarpTab; q += 32) s_tk[wid][q] = 0;   // tag 0: empty for every vertex
     if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
     __syncthreads();
     uint32_t tag = 0;
