@@ -11,6 +11,7 @@ ap.add_argument("--config", default="web_40m_2200m")
 ap.add_argument("--weights", default="ones")
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--async-too", action="store_true")
+ap.add_argument("--capture", default="", help="A or B: one synchronous sweep inside cudaProfilerStart/Stop (ncu --profile-from-start off)")
 a = ap.parse_args()
 g = synth.make(a.config, device="cuda")
 w = torch.ones(g.M, dtype=torch.float32, device="cuda") if a.weights == "ones" else None
@@ -21,6 +22,15 @@ Lconv = gg.labels().clone()
 ones = torch.ones(g.N, dtype=torch.uint8, device="cuda")
 Linit = torch.arange(g.N, dtype=torch.int32, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+if a.capture:
+    L = Linit if a.capture == "A" else Lconv
+    gg.set_labels(L, ones)
+    torch.cuda.synchronize()
+    torch.cuda.profiler.start()
+    gg.sweep(a.capture == "A", mode=nl.SYNC)
+    torch.cuda.synchronize()
+    torch.cuda.profiler.stop()
+    sys.exit(0)
 modes = [("sync", nl.SYNC)] + ([("async", nl.ASYNC)] if a.async_too else [])
 for name, L in (("A:init", Linit), ("B:converged", Lconv)):
     for mname, mode in modes:
