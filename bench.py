@@ -267,14 +267,17 @@ def run_ours(args):
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         t = json.load(open(tf))
-        if t.get("workload") == args.config and t.get("weights") == args.weights and t.get("kernel") == f"k_{BINS[dom]}":
-            # DRAM bytes per launch from ncu (dram__bytes_read.sum + dram__bytes_write.sum),
-            # compared with the algorithmic bytes per launch below
-            traffic = t["dram_bytes_per_launch"]
+        if t.get("workload") == args.config and t.get("weights") == args.weights and t.get("bin") == BINS[dom]:
+            # DRAM bytes per sweep of the bin from ncu (dram__bytes_read.sum +
+            # dram__bytes_write.sum of its kernels), compared with the
+            # algorithmic bytes per sweep below
+            traffic = t["dram_bytes_per_sweep"]
+    sweeps = sum(s["iterations"] for s in stats)
+    kname = {"warp": "k_frontier + k_warp"}.get(BINS[dom], f"k_{BINS[dom]}")
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": f"k_{BINS[dom]} (bin {BINS[dom]})",
-            "algorithmic_bytes_per_launch": int(byts / max(1, sum(s["launches"][dom] for s in stats))),
-            "traffic_source": "profiles/traffic.json (ncu, per k_warp launch)" if traffic else None,
+            "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": f"{kname} (bin {BINS[dom]})",
+            "algorithmic_bytes_per_sweep": int(byts / max(1, sweeps)),
+            "traffic_source": "profiles/traffic.json (ncu, per sweep of the bin's kernels)" if traffic else None,
             "peak_source": peak_src,
             "share_of_step": round(tot_ms[dom] / (ms * args.steps), 4),
             "algorithmic_bytes_per_run": int(byts / args.steps),

@@ -13,11 +13,12 @@
 //   giant tables: int32 keys / float32 values / int32 occupied-slot lists,
 //   one region of p1 = nextPow2(D)-1 slots per giant vertex.
 //
-// Kernels of one sweep (lpaMove), launched on the handle's stream in order
-// giant -> block -> warp -> thread (largest work first):
+// Kernels of one sweep (lpaMove), launched on the handle's stream, by default
+// in the order thread -> warp -> block -> giant (bin_order 1, hubs last):
 //   k_giant_snapshot / k_giant_accumulate / k_giant_reduce / k_giant_decide / k_giant_mark
 //   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
-//   k_warp    one warp per vertex, shared-memory table (<= 255 slots)
+//   k_frontier + k_warp   compacted frontier; one warp per vertex, pipelined,
+//                         shared-memory table (<= 511 slots)
 //   k_thread  one thread per vertex, labels in registers (degree < 32)
 
 #include "nulpa.h"
@@ -25,6 +26,8 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <type_traits>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -37,14 +40,9 @@ constexpr int32_t kEmpty = -1;           // phi
 constexpr int kMaxRetries = 16;          // R5
 constexpr int kMaxIter = 64;             // counters kept per iteration
 constexpr int kCtr = 24;                 // counters per iteration
+constexpr int kCtrRecs = 20;             // counter slot: warp-bin frontier size
 // counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
 
-constexpr int kWarpThreads = 256;        // k_warp: 8 warps per CTA
-constexpr int kWarpTab = 256;            // slots of a k_warp table (P1 = 255)
-#ifndef NULPA_WARP_CTAS
-#define NULPA_WARP_CTAS 6
-#endif
-constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;  // resident k_warp CTAs per SM (register budget)
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
 constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
 constexpr int kGiantChunk = 4096;        // edges per giant chunk
@@ -255,87 +253,24 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
     return x;
 }
 
-// Warp-private TAGGED table (k_warp): slot s holds tk[s] = (tag << 32) | key
-// and tv[s]; a slot whose tag is not the current vertex's tag is empty (phi),
-// so a table never needs hashtableClear -- every vertex gets a fresh tag.
-// B200 design change: the table lives in shared memory and is reused by all
-// vertices the warp processes, so its capacity P1 = 511 (p2 = 1023) is set by
-// the shared-memory budget instead of nextPow2(D)-1 (PAPER.md:208 sizes the
-// per-vertex GLOBAL tables that way; the giant bin keeps that sizing).  At
-// degree < 256 the load factor stays below 1/2, so probes rarely collide.
-// tt_add is Algorithm 2's accumulate (hybrid quadratic-double probing from
-// slot k mod p1, R5 linear continuation) for a leader adding its group's
-// weight x; it returns the label's new total.  Keys within one batch are
-// distinct (one leader per label), batches are ordered by __syncwarp, so the
-// value update is a plain read-modify-write; only the slot claim is atomic
-// (64-bit shared-memory CAS).
+// Shared-memory accessors with 32-bit shared-window addresses (the k_warp
+// tables); "memory" clobbers keep table reads/writes in program order.
 __device__ __forceinline__ uint64_t lds_u64(uint32_t addr) {
     uint64_t v;
     asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(addr) : "memory");
     return v;
 }
-__device__ __forceinline__ float lds_f32(uint32_t addr) {
-    float v;
-    asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
-    return v;
-}
 __device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
     asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 }
-__device__ __forceinline__ uint64_t cas_u64(uint32_t addr, uint64_t cmp, uint64_t val) {
-    uint64_t old;
-    asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "r"(addr), "l"(cmp), "l"(val) : "memory");
+__device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
+    // two empty slots: key = phi (0xFFFFFFFF), value = 0.0f
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %1, %2};" ::"r"(addr), "r"(0xFFFFFFFFu), "r"(0u) : "memory");
+}
+__device__ __forceinline__ uint32_t cas_u32(uint32_t addr, uint32_t cmp, uint32_t val) {
+    uint32_t old;
+    asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(addr), "r"(cmp), "r"(val) : "memory");
     return old;
-}
-
-// Full probe sequence (collisions, lost claim races): out of line.
-template <uint32_t P1>
-__device__ __noinline__ float tt_add_slow(uint32_t tk, uint32_t tv, uint32_t tag, int32_t k, float x) {
-    constexpr uint32_t p1 = P1, p2 = 2 * P1 + 1;
-    const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
-    uint32_t i = (uint32_t)k % p1, di = 1;
-    const uint32_t km = ((uint32_t)k % p2) % p1;           // 2nd hash
-    for (int t = 0;; ++t) {
-        const uint64_t cur = lds_u64(tk + 8 * i);
-        if (cur == want) {
-            const float V = __fadd_rn(lds_f32(tv + 4 * i), x);
-            sts_f32(tv + 4 * i, V);
-            return V;
-        }
-        if ((uint32_t)(cur >> 32) != tag && cas_u64(tk + 8 * i, cur, want) == cur) {   // empty: claim
-            sts_f32(tv + 4 * i, x);
-            return x;
-        }
-        if (t < kMaxRetries) {
-            i += di;
-            if (i >= p1) i -= p1;
-            di = 2 * di + km;
-            if (di >= p1) di -= p1;
-            if (di >= p1) di -= p1;
-        } else {
-            i = i + 1 == p1 ? 0 : i + 1;                   // R5
-        }
-    }
-}
-
-// Algorithm 2's accumulate into a warp-private tagged table at shared
-// addresses tk (keys, 8 B/slot) / tv (values, 4 B/slot).  Fast path: the
-// home slot k mod p1 holds (tag, k) or is free (stale tag) and is claimed.
-template <uint32_t P1>
-__device__ __forceinline__ float tt_add(uint32_t tk, uint32_t tv, uint32_t tag, int32_t k, float x) {
-    const uint64_t want = ((uint64_t)tag << 32) | (uint32_t)k;
-    const uint32_t i = (uint32_t)k % P1;
-    const uint64_t cur = lds_u64(tk + 8 * i);
-    if (cur == want) {
-        const float V = __fadd_rn(lds_f32(tv + 4 * i), x);
-        sts_f32(tv + 4 * i, V);
-        return V;
-    }
-    if ((uint32_t)(cur >> 32) != tag && cas_u64(tk + 8 * i, cur, want) == cur) {
-        sts_f32(tv + 4 * i, x);
-        return x;
-    }
-    return tt_add_slow<P1>(tk, tv, tag, k, x);
 }
 
 // One 32-edge batch of a warp against a table shared by several warps (the
@@ -505,160 +440,329 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
 }
 
 // ---------------------------------------------------------------------------
-// warp-per-vertex kernel: one 32-lane warp per vertex, the vertex's table
-// (p1 <= 255 slots) in shared memory, persistent grid-stride over the bin.
+// k_warp's per-vertex hashtable: one warp-private table in shared memory,
+// reused by every vertex the warp processes.  Capacity by degree class,
+// p1 in {255, 511} (a Mersenne number as in R1/R3, load factor <= 1/4 for
+// D < 64 and <= 1/2 above; PAPER.md:208 sizes per-vertex GLOBAL tables
+// p1 = nextPow2(D)-1 -- the giant bin keeps that sizing).  One 64-bit word
+// per slot (key | float value), so a probe is ONE ld.shared.b64; the table
+// is cleared with 16-byte stores before each vertex (hashtableClear,
+// PAPER.md:333).  Keys within one 32-entry batch are distinct (one leader per
+// label, match_any), batches are ordered by __syncwarp, so the value update
+// is a plain read-modify-write; only the slot claim is atomic.
 // ---------------------------------------------------------------------------
-template <bool SYNC, bool W, int TIE>
-__global__ void __launch_bounds__(kWarpThreads, kWarpCtasPerSm) k_warp(SweepArgs a, const int32_t *__restrict__ list,
-                                                          int64_t n) {
-    __shared__ uint64_t s_tk[kWarpThreads / 32][kWarpTab];   // static: 32-bit shared addressing
-    __shared__ float s_tv[kWarpThreads / 32][kWarpTab];
-    __shared__ unsigned long long bctr[4];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const uint32_t tk = (uint32_t)__cvta_generic_to_shared(&s_tk[wid][0]);
-    const uint32_t tv = (uint32_t)__cvta_generic_to_shared(&s_tv[wid][0]);
-    for (int q = lane; q < kWarpTab; q += 32) s_tk[wid][q] = 0;   // tag 0: empty for every vertex
-    if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
-    __syncthreads();
-    uint32_t tag = 0;
-    unsigned long long c_act = 0, c_edges = 0, c_ch = 0, c_che = 0;   // lane 0's tallies
-    const int64_t nw = (int64_t)gridDim.x * (kWarpThreads / 32);
-    const int64_t nchunks = (n + 31) / 32;
-    // Each warp takes chunks of 32 consecutive bin entries: the metadata of
-    // all 32 vertices (row, flag, offsets, own label) is fetched in one
-    // round trip, lane k holding vertex k; the warp then walks the active ones.
-    for (int64_t c = (int64_t)blockIdx.x * (kWarpThreads / 32) + wid; c < nchunks; c += nw) {
-        const int64_t t = c * 32 + lane;
-        int32_t r = 0, ci = 0;
-        int f = 0;
-        int64_t o = 0;
-        uint32_t deg = 0;
-        if (t < n) {
-            r = list[t];
-            f = a.flag_in[r + a.row_begin];
+constexpr int kWarpSlots = 512;          // largest class: p1 = 511
+
+// Algorithm 2's probe sequence past the home slot (hybrid quadratic-double
+// probing, R5 linear continuation) on a one-word-per-slot table of capacity P.
+template <uint32_t P>
+__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x) {
+    constexpr uint32_t p2 = 2 * P + 1;                    // R3
+    uint32_t i = (uint32_t)k % P, di = 1;
+    const uint32_t km = ((uint32_t)k % p2) % P;
+    for (int t = 1;; ++t) {
+        if (t <= kMaxRetries) {
+            i += di;
+            if (i >= P) i -= P;
+            di = 2 * di + km;
+            if (di >= P) di -= P;
+            if (di >= P) di -= P;
+        } else {
+            i = i + 1 == P ? 0 : i + 1;                    // R5
         }
-        if (f) {
-            o = a.offsets[r];
-            deg = (uint32_t)(a.offsets[r + 1] - o);
-            ci = a.lab_in[r + a.row_begin];
-            if (!SYNC) a.flag_in[r + a.row_begin] = 0;     // mark i as processed
+        const uint64_t cur = lds_u64(tab + 8 * i);
+        const int32_t ck = (int32_t)(uint32_t)cur;
+        if (ck == k) {
+            const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
+            sts_f32(tab + 8 * i + 4, V);
+            return V;
         }
-        unsigned act = __ballot_sync(0xFFFFFFFFu, f != 0);
-        while (act) {
-            const int k = __ffs(act) - 1;
-            act &= act - 1;
-            const int32_t rk = __shfl_sync(0xFFFFFFFFu, r, k);
-            const int64_t ok = __shfl_sync(0xFFFFFFFFu, o, k);
-            const uint32_t dk = __shfl_sync(0xFFFFFFFFu, deg, k);
-            const int32_t cik = __shfl_sync(0xFFFFFFFFu, ci, k);
-            const int64_t vk = rk + a.row_begin;
-            Hash h;
-            h.init(dk);
-            TieOrder<TIE> to;
-            to.init(h);
-            // the first 64 entries of the row stay in registers; indices and
-            // weights first, then all the neighbour labels
-            const bool v0 = (uint32_t)lane < dk, v1 = (uint32_t)(lane + 32) < dk;
-            const int32_t j0 = v0 ? __ldcs(a.indices + ok + lane) : -1;
-            const int32_t j1 = v1 ? __ldcs(a.indices + ok + 32 + lane) : -1;
-            float w0 = 0.0f, w1 = 0.0f;
-            if (W) {
-                if (v0) w0 = __ldcs(a.weights + ok + lane);
-                if (v1) w1 = __ldcs(a.weights + ok + 32 + lane);
-            }
-            const int32_t k0 = (j0 >= 0 && j0 != (int32_t)vk) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
-            const int32_t k1 = (j1 >= 0 && j1 != (int32_t)vk) ? a.lab_in[j1] : kEmpty;
-            // per-lane running best (weight bits + 1, label) over the label
-            // totals this lane produced as a group leader; the maximum over
-            // all lanes is hashtableMaxKey (totals only grow, so partial
-            // totals never exceed the final maximum)
-            uint32_t bw = 0;
-            int32_t bk = 0;
-            auto offer = [&](float V, int32_t key) {
-                const uint32_t vb = __float_as_uint(V) + 1;
-                if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
-                    bw = vb;
-                    bk = key;
-                }
-            };
-            auto fold = [&](int32_t key, float w, unsigned &grp) -> float {
-                grp = __match_any_sync(0xFFFFFFFFu, key);
-                if (W) {
-                    // all weights of the batch equal (e.g. the paper's default
-                    // weight 1): the group total is count * w, the correctly
-                    // rounded sum (exact for integer-valued weights)
-                    const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
-                    if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
-                    const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-                    return maxn > 1 ? group_sum(grp, w, maxn) : w;
-                }
-                return (float)__popc(grp);
-            };
-            if (dk <= 32) {
-                // one batch: the match_any groups ARE the label totals -- no table
-                unsigned grp;
-                const float x = fold(k0, w0, grp);
-                if (k0 != kEmpty && lane == __ffs(grp) - 1) offer(x, k0);
-            } else {
-                ++tag;
-                auto batch = [&](int32_t key, float w) {
-                    unsigned grp;
-                    const float x = fold(key, w, grp);
-                    if (key != kEmpty && lane == __ffs(grp) - 1) offer(tt_add<kWarpTab - 1>(tk, tv, tag, key, x), key);
-                    __syncwarp();
-                };
-                batch(k0, w0);
-                batch(k1, w1);
-                for (uint32_t b = 64; b < dk; b += 64) {
-                    const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
-                    const int32_t i0 = u0 ? __ldcs(a.indices + ok + b + lane) : -1;
-                    const int32_t i1 = u1 ? __ldcs(a.indices + ok + b + 32 + lane) : -1;
-                    float x0 = 0.0f, x1 = 0.0f;
-                    if (W) {
-                        if (u0) x0 = __ldcs(a.weights + ok + b + lane);
-                        if (u1) x1 = __ldcs(a.weights + ok + b + 32 + lane);
-                    }
-                    const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
-                    const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
-                    batch(q0, x0);
-                    if (b + 32 < dk) batch(q1, x1);
-                }
-            }
-            // hashtableMaxKey: max weight, then first label in tie order
-            const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
-            int32_t cs = kEmpty;
-            if (W1) {
-                const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
-                cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
-            }
-            const bool changed = accept_move(cs, cik, a.pickless);
-            if (changed) {
-                if (lane == 0) a.lab_out[vk] = cs;
-                if (j0 >= 0) a.flag_out[j0] = 1;            // mark neighbours unprocessed
-                if (j1 >= 0) a.flag_out[j1] = 1;
-                for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[a.indices[ok + b]] = 1;
-            }
-            c_act += 1;
-            c_edges += dk;
-            c_ch += changed;
-            c_che += changed ? dk : 0;
+        if (ck == kEmpty && cas_u32(tab + 8 * i, 0xFFFFFFFFu, (uint32_t)k) == 0xFFFFFFFFu) {
+            sts_f32(tab + 8 * i + 4, x);
+            return x;
         }
     }
+}
+
+// hashtableAccumulate (Algorithm 2) for a leader adding its group's weight x
+// to label k; keys of one batch are distinct, so only the claim is atomic.
+// Returns the label's new total.
+template <uint32_t P>
+__device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, float x) {
+    const uint32_t i = (uint32_t)k % P;
+    const uint64_t cur = lds_u64(tab + 8 * i);
+    const int32_t ck = (int32_t)(uint32_t)cur;
+    if (ck == k) {
+        const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
+        sts_f32(tab + 8 * i + 4, V);
+        return V;
+    }
+    if (ck == kEmpty && cas_u32(tab + 8 * i, 0xFFFFFFFFu, (uint32_t)k) == 0xFFFFFFFFu) {
+        sts_f32(tab + 8 * i + 4, x);
+        return x;
+    }
+    return kv_add_slow<P>(tab, k, x);
+}
+
+// ---------------------------------------------------------------------------
+// Frontier compaction (vertex pruning, "if not unprocessed(i)
+// continue; mark i as processed"): one pass over a bin list writes a 16-byte
+// record {offset, degree, row, C[i]} per unprocessed vertex and clears its
+// flag (async).  The warp kernel then streams records at known addresses, so
+// the loads of upcoming vertices can be issued ahead (software pipelining)
+// instead of waiting on list -> flag -> offsets dependent round trips.
+// C[i] read here is still C[i] when i is processed: only i writes C[i].
+// Also counts processed vertices and their edges (counters 1+bin, 5+bin).
+// ---------------------------------------------------------------------------
+struct __align__(16) VRec {
+    uint32_t o_lo;      // offsets[r], low 32 bits
+    uint32_t o_hi_deg;  // offsets[r] bits 32..47 | degree << 16 (degree < 2^16 in the warp bin)
+    int32_t r;          // local row
+    int32_t ci;         // C[i]
+};
+
+template <bool SYNC>
+__global__ void __launch_bounds__(256) k_frontier(SweepArgs a, const int32_t *__restrict__ list, int64_t n, int bin,
+                                                  VRec *__restrict__ recs, unsigned long long *count) {
+    __shared__ unsigned long long bctr[2];
+    if (threadIdx.x < 2) bctr[threadIdx.x] = 0;
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    uint32_t c_act = 0;
+    unsigned long long c_edges = 0;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
+        const int64_t t = base + lane;
+        int f = 0;
+        VRec rec;
+        uint32_t deg = 0;
+        if (t < n) {
+            const int32_t r = list[t];
+            const int64_t v = r + a.row_begin;
+            f = a.flag_in[v];
+            if (f) {
+                const int64_t o = a.offsets[r];
+                deg = (uint32_t)(a.offsets[r + 1] - o);
+                rec.o_lo = (uint32_t)o;
+                rec.o_hi_deg = (uint32_t)((uint64_t)o >> 32) | (deg << 16);
+                rec.r = r;
+                rec.ci = a.lab_in[v];
+                if (!SYNC) a.flag_in[v] = 0;              // mark i as processed
+            }
+        }
+        const unsigned m = __ballot_sync(0xFFFFFFFFu, f != 0);
+        unsigned long long pos = 0;
+        if (lane == 0 && m) pos = atomicAdd(count, (unsigned long long)__popc(m));
+        pos = __shfl_sync(0xFFFFFFFFu, pos, 0);
+        if (f) recs[pos + __popc(m & ((1u << lane) - 1))] = rec;
+        c_act += __popc(m);
+        c_edges += __reduce_add_sync(0xFFFFFFFFu, deg);
+    }
     if (lane == 0 && c_act) {
-        atomicAdd(&bctr[0], c_act);
+        atomicAdd(&bctr[0], (unsigned long long)c_act);
         atomicAdd(&bctr[1], c_edges);
-        atomicAdd(&bctr[2], c_ch);
-        atomicAdd(&bctr[3], c_che);
     }
     __syncthreads();
     if (threadIdx.x == 0 && bctr[0]) {
-        atomicAdd(&a.ctr[1 + 1], bctr[0]);
-        atomicAdd(&a.ctr[5 + 1], bctr[1]);
-        if (bctr[2]) {
-            atomicAdd(&a.ctr[0], bctr[2]);
-            atomicAdd(&a.ctr[9 + 1], bctr[2]);
-            atomicAdd(&a.ctr[13 + 1], bctr[3]);
+        atomicAdd(&a.ctr[1 + bin], bctr[0]);
+        atomicAdd(&a.ctr[5 + bin], bctr[1]);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// warp-per-vertex kernel (switch_degree <= D < block_degree), over the
+// compacted frontier and software-pipelined across the vertices of a warp.
+// A warp owns record groups gw, gw + nw, ... (32 records each) and walks them
+// as one sequence n = 0, 1, ...; while vertex n is folded, the label gathers
+// of vertex n+1 and the index/weight loads of vertex n+2 are in flight, so
+// each dependent global round trip overlaps a whole vertex of work.  Records
+// reach shared memory one group ahead (a 2-group ring per warp).
+// Per 32-entry batch: match_any folds lanes holding the same label onto a
+// leader, whose group total (count * w when the batch's weights are all
+// equal, else a pairwise tree) is added into the table (Algorithm 2); each
+// lane keeps the best (total, label) it produced as a leader, and two
+// redux.max give hashtableMaxKey without scanning the table.  Degree <= 32
+// needs no table (the match groups are the totals).
+// Asynchronous reading: vertex n+1's neighbour labels are gathered before
+// vertex n's new label is written; the gathered copies of that label are
+// patched in registers, so n+1 still sees n's move.
+// ---------------------------------------------------------------------------
+constexpr int kWarpWarps = 8;            // warps per CTA
+#ifndef NULPA_WARP_CTAS
+#define NULPA_WARP_CTAS 4
+#endif
+constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
+
+template <bool SYNC, bool W, int TIE>
+__global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepArgs a, const VRec *__restrict__ recs,
+                                                                        const unsigned long long *__restrict__ count) {
+    __shared__ __align__(16) uint64_t s_tab[kWarpWarps][kWarpSlots];
+    __shared__ VRec s_ring[kWarpWarps][2][32];
+    __shared__ unsigned long long bctr[2];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const uint32_t tab = (uint32_t)__cvta_generic_to_shared(&s_tab[wid][0]);
+    if (threadIdx.x < 2) bctr[threadIdx.x] = 0;
+    __syncthreads();
+    const int64_t nrec = (int64_t)*count;
+    const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
+    const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
+    const int64_t ng = (nrec + 31) / 32;
+    const int64_t nq = gw < ng ? (ng - 1 - gw) / nw + 1 : 0;            // groups of this warp
+    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - (gw + (nq - 1) * nw) * 32) : 0;
+    unsigned long long c_ch = 0, c_che = 0;
+    auto grec = [&](int64_t q) -> VRec {                   // lane's record of group q (or empty)
+        VRec z{0, 0, 0, 0};
+        const int64_t i = (gw + q * nw) * 32 + lane;
+        return (q < nq && i < nrec) ? recs[i] : z;
+    };
+    auto rrec = [&](int64_t m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
+    auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
+    auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
+    if (nv) {
+        s_ring[wid][0][lane] = grec(0);
+        s_ring[wid][1][lane] = grec(1);
+    }
+    VRec pend = grec(2);
+    __syncwarp();
+    // pipeline registers: stage 2 (indices/weights issued), stage 1 (labels issued), stage 0 (fold)
+    int32_t j2a = -1, j2b = -1, j1a = -1, j1b = -1, j0a = -1, j0b = -1;
+    float w2a = 1.0f, w2b = 1.0f, w1a = 1.0f, w1b = 1.0f, w0a = 1.0f, w0b = 1.0f;
+    int32_t k1a = kEmpty, k1b = kEmpty, k0a = kEmpty, k0b = kEmpty;
+    auto load_row = [&](int64_t m, int32_t &ja, int32_t &jb, float &wa, float &wb) {
+        ja = jb = -1;
+        wa = wb = 1.0f;
+        if (m < nv) {
+            const VRec r = rrec(m);
+            const uint32_t d = r_d(r);
+            const int64_t o = r_o(r);
+            if ((uint32_t)lane < d) ja = __ldcs(a.indices + o + lane);
+            if ((uint32_t)lane + 32 < d) jb = __ldcs(a.indices + o + 32 + lane);
+            if (W) {
+                if ((uint32_t)lane < d) wa = __ldcs(a.weights + o + lane);
+                if ((uint32_t)lane + 32 < d) wb = __ldcs(a.weights + o + 32 + lane);
+            }
         }
+    };
+    auto gather = [&](int64_t m, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
+        ka = kb = kEmpty;
+        if (m < nv) {
+            const int32_t vk = (int32_t)(rrec(m).r + a.row_begin);
+            if (ja >= 0 && ja != vk) ka = a.lab_in[ja];     // "if j = i continue"
+            if (jb >= 0 && jb != vk) kb = a.lab_in[jb];
+        }
+    };
+    load_row(0, j0a, j0b, w0a, w0b);
+    load_row(1, j1a, j1b, w1a, w1b);
+    gather(0, j0a, j0b, k0a, k0b);
+    for (int64_t n = 0; n < nv; ++n) {
+        if ((n & 31) == 0 && n > 0) {
+            // entering group q = n/32: group q+1 goes where group q-1 was, group q+2 is requested
+            s_ring[wid][((n >> 5) + 1) & 1][lane] = pend;
+            pend = grec((n >> 5) + 2);
+            __syncwarp();
+        }
+        load_row(n + 2, j2a, j2b, w2a, w2b);
+        gather(n + 1, j1a, j1b, k1a, k1b);
+        // ---- fold vertex n ----
+        const VRec rc = rrec(n);
+        const uint32_t dk = r_d(rc);
+        const int64_t ok = r_o(rc);
+        const int64_t vk = rc.r + a.row_begin;
+        Hash h;
+        h.init(dk);
+        TieOrder<TIE> to;
+        to.init(h);
+        uint32_t bw = 0;
+        int32_t bk = 0;
+        auto offer = [&](float V, int32_t key) {
+            const uint32_t vb = __float_as_uint(V) + 1;
+            if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
+                bw = vb;
+                bk = key;
+            }
+        };
+        auto fold = [&](int32_t key, float w, bool &leader) -> float {
+            const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+            leader = key != kEmpty && (grp & ((1u << lane) - 1)) == 0;
+            if (W) {
+                const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
+                if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
+                const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+                return maxn > 1 ? group_sum(grp, w, maxn) : w;
+            }
+            return (float)__popc(grp);
+        };
+        const int32_t *pi = a.indices + ok + lane;
+        const float *pw = W ? a.weights + ok + lane : nullptr;
+        auto table_row = [&](auto cap) {
+            constexpr uint32_t P = decltype(cap)::value;
+#pragma unroll
+            for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
+            __syncwarp();
+            auto batch = [&](int32_t key, float w) {
+                bool leader;
+                const float x = fold(key, w, leader);
+                if (leader) offer(kv_add<P>(tab, key, x), key);
+                __syncwarp();
+            };
+            batch(k0a, w0a);
+            batch(k0b, w0b);
+            for (uint32_t b = 64; b < dk; b += 64) {
+                const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
+                const int32_t i0 = u0 ? __ldcs(pi + b) : -1;
+                const int32_t i1 = u1 ? __ldcs(pi + b + 32) : -1;
+                float x0 = 1.0f, x1 = 1.0f;
+                if (W) {
+                    if (u0) x0 = __ldcs(pw + b);
+                    if (u1) x1 = __ldcs(pw + b + 32);
+                }
+                const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
+                const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
+                batch(q0, x0);
+                if (b + 32 < dk) batch(q1, x1);
+            }
+        };
+        if (dk <= 32) {
+            bool leader;
+            const float x = fold(k0a, w0a, leader);
+            if (leader) offer(x, k0a);
+        } else if (dk < 64) {
+            table_row(std::integral_constant<uint32_t, 255>());
+        } else {
+            table_row(std::integral_constant<uint32_t, 511>());
+        }
+        const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
+        int32_t cs = kEmpty;
+        if (W1) {
+            const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
+            cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
+        }
+        if (accept_move(cs, rc.ci, a.pickless)) {
+            c_ch += 1;
+            c_che += dk;
+            if (lane == 0) a.lab_out[vk] = cs;
+            if (!SYNC) {
+                // vertex n+1's labels were gathered before this write: patch them
+                if (j1a == (int32_t)vk) k1a = cs;
+                if (j1b == (int32_t)vk) k1b = cs;
+            }
+            if (j0a >= 0) a.flag_out[j0a] = 1;            // mark neighbours unprocessed
+            if (j0b >= 0) a.flag_out[j0b] = 1;
+            for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[pi[b - lane]] = 1;
+        }
+        // rotate the pipeline
+        j0a = j1a; j0b = j1b; w0a = w1a; w0b = w1b; k0a = k1a; k0b = k1b;
+        j1a = j2a; j1b = j2b; w1a = w2a; w1b = w2b;
+    }
+    if (lane == 0 && c_ch) {
+        atomicAdd(&bctr[0], c_ch);
+        atomicAdd(&bctr[1], c_che);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && bctr[0]) {
+        atomicAdd(&a.ctr[0], bctr[0]);
+        atomicAdd(&a.ctr[9 + 1], bctr[0]);
+        atomicAdd(&a.ctr[13 + 1], bctr[1]);
     }
 }
 
@@ -1248,6 +1352,7 @@ struct nulpa_graph {
     int32_t t1 = 0, t2 = 0, t3 = 0;
     bool bins_built = false;
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
+    void *wrecs = nullptr;          // warp-bin frontier records (VRec [bin_n[1]])
     int64_t bin_n[4] = {0, 0, 0, 0};
     int64_t bin_e[4] = {0, 0, 0, 0};
     int64_t bin_maxdeg[4] = {0, 0, 0, 0};
@@ -1291,6 +1396,8 @@ int dalloc(T **p, size_t n) {
 }
 
 void free_bins(nulpa_graph *g) {
+    cudaFree(g->wrecs);
+    g->wrecs = nullptr;
     for (int b = 0; b < 4; ++b) {
         cudaFree(g->bin_list[b]);
         g->bin_list[b] = nullptr;
@@ -1542,9 +1649,12 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[1];
         CHECK(rec(1, 0));
         if (n > 0) {
-            k_warp<SYNC, W, TIE><<<grid_for((n + 31) / 32, kWarpThreads / 32, sms * kWarpCtasPerSm), kWarpThreads, 0, cs>>>(a, g->bin_list[1], n);
+            if (!g->wrecs) CHECK(dalloc(reinterpret_cast<VRec **>(&g->wrecs), (size_t)n));
+            VRec *recs = reinterpret_cast<VRec *>(g->wrecs);
+            k_frontier<SYNC><<<grid_for(n, 256, sms * 8), 256, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs);
+            k_warp<SYNC, W, TIE><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs);
             CU(cudaGetLastError());
-            g->stats.launches[1] += 1;
+            g->stats.launches[1] += 2;
         }
         CHECK(rec(1, 1));
         return NULPA_OK;
@@ -1700,6 +1810,7 @@ int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *we
     }
     if (M < 0) return bail(fail(NULPA_EINVAL, "offsets[n_rows] must be >= 0"));
     if (M > 0 && !indices) return bail(fail(NULPA_EINVAL, "indices is NULL"));
+    if (M >= (INT64_C(1) << 48)) return bail(fail(NULPA_EINVAL, "more than 2^48 CSR entries"));
     g->M = M;
     if (memkind == NULPA_MEM_DEVICE) {
         g->offsets = const_cast<int64_t *>(offsets);

@@ -1,6 +1,7 @@
 """profiles/traffic.json from an ncu launch list with dram__bytes_read/write
 (`ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum
--k regex:^k_ --csv --log-file X python bench.py ...`)."""
+-k regex:^k_ --csv --log-file X python bench.py ...`): DRAM bytes per sweep of
+the warp bin (one k_frontier + one k_warp launch per sweep)."""
 import csv, collections, json, sys
 path, workload, weights = sys.argv[1], sys.argv[2], sys.argv[3]
 rows = [r for r in csv.reader(open(path)) if r]
@@ -14,10 +15,15 @@ for r in rows[hi + 1:]:
         continue
     per[r[iid]][r[im]] = float(r[iv].replace(",", ""))
     name[r[iid]] = r[ik]
-warp = [d for k, d in per.items() if "k_warp" in name[k]]
-b = [d["dram__bytes_read.sum"] + d["dram__bytes_write.sum"] for d in warp]
-out = {"workload": workload, "weights": weights, "kernel": "k_warp", "launches": len(b),
-       "dram_bytes_per_launch": sum(b) / len(b), "per_launch": b,
+def dram(k):
+    return per[k]["dram__bytes_read.sum"] + per[k]["dram__bytes_write.sum"]
+warp = [k for k in per if "k_warp" in name[k]]
+front = [k for k in per if "k_frontier" in name[k]]
+assert len(warp) == len(front), (len(warp), len(front))
+b = [dram(f) + dram(w) for f, w in zip(front, warp)]
+out = {"workload": workload, "weights": weights, "bin": "warp", "kernels": ["k_frontier", "k_warp"],
+       "sweeps": len(b), "dram_bytes_per_sweep": sum(b) / len(b), "per_sweep": b,
+       "k_warp_per_launch": [dram(w) for w in warp], "k_frontier_per_launch": [dram(f) for f in front],
        "source": path, "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none (cold, serialised launches)"}
 json.dump(out, open("profiles/traffic.json", "w"), indent=1)
-print(out["dram_bytes_per_launch"] / 1e9, "GB per launch over", len(b), "launches")
+print(out["dram_bytes_per_sweep"] / 1e9, "GB per sweep over", len(b), "sweeps")
