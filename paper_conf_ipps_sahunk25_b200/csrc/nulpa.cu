@@ -615,23 +615,25 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
         const int64_t i = (gw + q * nw) * 32 + lane;
         return (q < nq && i < nrec) ? recs[i] : z;
     };
-    auto rrec = [&](int64_t m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
+    auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
     auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
-    if (nv) {
-        s_ring[wid][0][lane] = grec(0);
-        s_ring[wid][1][lane] = grec(1);
-    }
+    s_ring[wid][0][lane] = grec(0);                      // zero records (degree 0) past the end
+    s_ring[wid][1][lane] = grec(1);
     VRec pend = grec(2);
     __syncwarp();
-    // pipeline registers: stage 2 (indices/weights issued), stage 1 (labels issued), stage 0 (fold)
-    int32_t j2a = -1, j2b = -1, j1a = -1, j1b = -1, j0a = -1, j0b = -1;
-    float w2a = 1.0f, w2b = 1.0f, w1a = 1.0f, w1b = 1.0f, w0a = 1.0f, w0b = 1.0f;
-    int32_t k1a = kEmpty, k1b = kEmpty, k0a = kEmpty, k0b = kEmpty;
-    auto load_row = [&](int64_t m, int32_t &ja, int32_t &jb, float &wa, float &wb) {
+    // pipeline registers of one vertex: entries lane and lane+32 of its row
+    // (index j, weight w, neighbour label k)
+    struct Stage {
+        int32_t ja, jb;
+        float wa, wb;
+        int32_t ka, kb;
+    };
+    Stage SA{-1, -1, 1.0f, 1.0f, kEmpty, kEmpty}, SB = SA, SC = SA;
+    auto load_row = [&](int m, int32_t &ja, int32_t &jb, float &wa, float &wb) {
         ja = jb = -1;
         wa = wb = 1.0f;
-        if (m < nv) {
+        {   // past the end the ring holds zero records (degree 0): no loads
             const VRec r = rrec(m);
             const uint32_t d = r_d(r);
             const int64_t o = r_o(r);
@@ -643,26 +645,28 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
             }
         }
     };
-    auto gather = [&](int64_t m, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
+    auto gather = [&](int m, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
         ka = kb = kEmpty;
-        if (m < nv) {
+        {
             const int32_t vk = (int32_t)(rrec(m).r + a.row_begin);
             if (ja >= 0 && ja != vk) ka = a.lab_in[ja];     // "if j = i continue"
             if (jb >= 0 && jb != vk) kb = a.lab_in[jb];
         }
     };
-    load_row(0, j0a, j0b, w0a, w0b);
-    load_row(1, j1a, j1b, w1a, w1b);
-    gather(0, j0a, j0b, k0a, k0b);
-    for (int64_t n = 0; n < nv; ++n) {
+    load_row(0, SA.ja, SA.jb, SA.wa, SA.wb);
+    load_row(1, SB.ja, SB.jb, SB.wa, SB.wb);
+    gather(0, SA.ja, SA.jb, SA.ka, SA.kb);
+    // one pipeline step: issue vertex n+2's row loads (s2), vertex n+1's label
+    // gathers (s1), fold vertex n (s0)
+    auto step = [&](int n, Stage &s0, Stage &s1, Stage &s2) {
         if ((n & 31) == 0 && n > 0) {
             // entering group q = n/32: group q+1 goes where group q-1 was, group q+2 is requested
             s_ring[wid][((n >> 5) + 1) & 1][lane] = pend;
             pend = grec((n >> 5) + 2);
             __syncwarp();
         }
-        load_row(n + 2, j2a, j2b, w2a, w2b);
-        gather(n + 1, j1a, j1b, k1a, k1b);
+        load_row(n + 2, s2.ja, s2.jb, s2.wa, s2.wb);
+        gather(n + 1, s1.ja, s1.jb, s1.ka, s1.kb);
         // ---- fold vertex n ----
         const VRec rc = rrec(n);
         const uint32_t dk = r_d(rc);
@@ -705,8 +709,8 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
                 if (leader) offer(kv_add<P>(tab, key, x), key);
                 __syncwarp();
             };
-            batch(k0a, w0a);
-            batch(k0b, w0b);
+            batch(s0.ka, s0.wa);
+            batch(s0.kb, s0.wb);
             for (uint32_t b = 64; b < dk; b += 64) {
                 const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
                 const int32_t i0 = u0 ? __ldcs(pi + b) : -1;
@@ -724,8 +728,8 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
         };
         if (dk <= 32) {
             bool leader;
-            const float x = fold(k0a, w0a, leader);
-            if (leader) offer(x, k0a);
+            const float x = fold(s0.ka, s0.wa, leader);
+            if (leader) offer(x, s0.ka);
         } else if (dk < 64) {
             table_row(std::integral_constant<uint32_t, 255>());
         } else {
@@ -743,16 +747,19 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
             if (lane == 0) a.lab_out[vk] = cs;
             if (!SYNC) {
                 // vertex n+1's labels were gathered before this write: patch them
-                if (j1a == (int32_t)vk) k1a = cs;
-                if (j1b == (int32_t)vk) k1b = cs;
+                if (s1.ja == (int32_t)vk) s1.ka = cs;
+                if (s1.jb == (int32_t)vk) s1.kb = cs;
             }
-            if (j0a >= 0) a.flag_out[j0a] = 1;            // mark neighbours unprocessed
-            if (j0b >= 0) a.flag_out[j0b] = 1;
+            if (s0.ja >= 0) a.flag_out[s0.ja] = 1;        // mark neighbours unprocessed
+            if (s0.jb >= 0) a.flag_out[s0.jb] = 1;
             for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[pi[b - lane]] = 1;
         }
-        // rotate the pipeline
-        j0a = j1a; j0b = j1b; w0a = w1a; w0b = w1b; k0a = k1a; k0b = k1b;
-        j1a = j2a; j1b = j2b; w1a = w2a; w1b = w2b;
+    };
+    // (unrolling by 3 so the stages rotate by renaming overflows the instruction cache: 30% slower)
+    for (int n = 0; n < (int)nv; ++n) {
+        step(n, SA, SB, SC);
+        SA = SB;
+        SB = SC;
     }
     if (lane == 0 && c_ch) {
         atomicAdd(&bctr[0], c_ch);
