@@ -72,6 +72,11 @@ typedef struct nulpa_params {
                                     within a sweep (hubs last); 0: giant, block, warp, thread;
                                     2: block + giant on a second stream, concurrent with
                                     thread + warp                                               */
+    int32_t wide_degree;         /* within the block bin: degree < this -> one warp per vertex
+                                    with a warp-private 1023-slot shared-memory table (load
+                                    <= 1/2); degree >= this -> one CTA per vertex.  Range
+                                    [1, 512]; <= block_degree sends the whole bin to the CTA
+                                    kernel.  B200 default 512                                   */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0

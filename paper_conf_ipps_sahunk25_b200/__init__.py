@@ -25,7 +25,8 @@ __all__ = [
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_PKG, "libnulpa.so")
+# NULPA_LIB: load another build of the library (kernel A/B experiments only)
+_LIB_PATH = os.environ.get("NULPA_LIB") or os.path.join(_PKG, "libnulpa.so")
 
 ASYNC, SYNC = 0, 1
 TIE_SMALLEST, TIE_SLOT = 0, 1
@@ -50,6 +51,7 @@ class Params(ctypes.Structure):
         ("timing", ctypes.c_int32),
         ("tie_rule", ctypes.c_int32),
         ("bin_order", ctypes.c_int32),
+        ("wide_degree", ctypes.c_int32),
     ]
 
 

@@ -41,6 +41,8 @@ constexpr int kMaxRetries = 16;          // R5
 constexpr int kMaxIter = 64;             // counters kept per iteration
 constexpr int kCtr = 24;                 // counters per iteration
 constexpr int kCtrRecs = 20;             // counter slot: warp-bin frontier size
+constexpr int kCtrRecsW = 21;            // counter slot: block-bin frontier, warp-per-vertex part
+constexpr int kCtrRecsB = 22;            // counter slot: block-bin frontier, CTA-per-vertex part
 // counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
 
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
@@ -521,43 +523,88 @@ struct __align__(16) VRec {
     int32_t ci;         // C[i]
 };
 
+// With a split degree (block bin): records of degree < split go to recs
+// (count), the others to recs2 (count2).  Positions are reserved with ONE
+// global atomic per CTA tile of kFrontTile list entries (a single counter
+// hit by one atomic per warp serialised ~1M atomics at L2: ~1 ms per sweep);
+// within a tile, records keep list (row) order.
+#ifndef NULPA_FRONT_PER
+#define NULPA_FRONT_PER 1
+#endif
+constexpr int kFrontThreads = 256, kFrontPer = NULPA_FRONT_PER, kFrontTile = kFrontThreads * kFrontPer;
 template <bool SYNC>
-__global__ void __launch_bounds__(256) k_frontier(SweepArgs a, const int32_t *__restrict__ list, int64_t n, int bin,
-                                                  VRec *__restrict__ recs, unsigned long long *count) {
+__global__ void __launch_bounds__(kFrontThreads) k_frontier(SweepArgs a, const int32_t *__restrict__ list, int64_t n,
+                                                           int bin, VRec *__restrict__ recs,
+                                                           unsigned long long *count, uint32_t split,
+                                                           VRec *__restrict__ recs2, unsigned long long *count2) {
+    constexpr int NW = kFrontThreads / 32;
+    __shared__ uint32_t s_c[2][NW];
+    __shared__ unsigned long long s_base[2];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    uint32_t c_act = 0;
+    unsigned long long c_edges = 0;
+    for (int64_t tile = (int64_t)blockIdx.x * kFrontTile; tile < n; tile += (int64_t)gridDim.x * kFrontTile) {
+        // warp w owns entries tile + w*32*kFrontPer + [0, 32*kFrontPer), in 32-entry rounds
+        VRec rec[kFrontPer];
+        unsigned m[kFrontPer], m2[kFrontPer];
+        uint32_t c1 = 0, c2 = 0;
+#pragma unroll
+        for (int k = 0; k < kFrontPer; ++k) {
+            const int64_t t = tile + (wid * kFrontPer + k) * 32 + lane;
+            int f = 0;
+            uint32_t deg = 0;
+            if (t < n) {
+                const int32_t r = list[t];
+                const int64_t v = r + a.row_begin;
+                f = a.flag_in[v];
+                if (f) {
+                    const int64_t o = a.offsets[r];
+                    deg = (uint32_t)(a.offsets[r + 1] - o);
+                    rec[k].o_lo = (uint32_t)o;
+                    rec[k].o_hi_deg = (uint32_t)((uint64_t)o >> 32) | (deg << 16);
+                    rec[k].r = r;
+                    rec[k].ci = a.lab_in[v];
+                    if (!SYNC) a.flag_in[v] = 0;          // mark i as processed
+                }
+            }
+            const bool hi = f && deg >= split;
+            m[k] = __ballot_sync(0xFFFFFFFFu, f && !hi);
+            m2[k] = __ballot_sync(0xFFFFFFFFu, hi);
+            c1 += __popc(m[k]);
+            c2 += __popc(m2[k]);
+            c_edges += __reduce_add_sync(0xFFFFFFFFu, deg);
+        }
+        c_act += c1 + c2;
+        if (lane == 0) {
+            s_c[0][wid] = c1;
+            s_c[1][wid] = c2;
+        }
+        __syncthreads();
+        if (threadIdx.x < 2) {
+            uint32_t tot = 0;
+#pragma unroll
+            for (int w = 0; w < NW; ++w) tot += s_c[threadIdx.x][w];
+            s_base[threadIdx.x] = tot ? atomicAdd(threadIdx.x ? count2 : count, (unsigned long long)tot) : 0;
+        }
+        __syncthreads();
+        unsigned long long p1 = s_base[0], p2 = s_base[1];
+        for (int w = 0; w < wid; ++w) {
+            p1 += s_c[0][w];
+            p2 += s_c[1][w];
+        }
+        __syncthreads();                                  // s_c / s_base reused by the next tile
+#pragma unroll
+        for (int k = 0; k < kFrontPer; ++k) {
+            const unsigned below = (1u << lane) - 1;
+            if (m[k] >> lane & 1) recs[p1 + __popc(m[k] & below)] = rec[k];
+            if (m2[k] >> lane & 1) recs2[p2 + __popc(m2[k] & below)] = rec[k];
+            p1 += __popc(m[k]);
+            p2 += __popc(m2[k]);
+        }
+    }
     __shared__ unsigned long long bctr[2];
     if (threadIdx.x < 2) bctr[threadIdx.x] = 0;
     __syncthreads();
-    const int lane = threadIdx.x & 31;
-    uint32_t c_act = 0;
-    unsigned long long c_edges = 0;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < n; base += stride) {
-        const int64_t t = base + lane;
-        int f = 0;
-        VRec rec;
-        uint32_t deg = 0;
-        if (t < n) {
-            const int32_t r = list[t];
-            const int64_t v = r + a.row_begin;
-            f = a.flag_in[v];
-            if (f) {
-                const int64_t o = a.offsets[r];
-                deg = (uint32_t)(a.offsets[r + 1] - o);
-                rec.o_lo = (uint32_t)o;
-                rec.o_hi_deg = (uint32_t)((uint64_t)o >> 32) | (deg << 16);
-                rec.r = r;
-                rec.ci = a.lab_in[v];
-                if (!SYNC) a.flag_in[v] = 0;              // mark i as processed
-            }
-        }
-        const unsigned m = __ballot_sync(0xFFFFFFFFu, f != 0);
-        unsigned long long pos = 0;
-        if (lane == 0 && m) pos = atomicAdd(count, (unsigned long long)__popc(m));
-        pos = __shfl_sync(0xFFFFFFFFu, pos, 0);
-        if (f) recs[pos + __popc(m & ((1u << lane) - 1))] = rec;
-        c_act += __popc(m);
-        c_edges += __reduce_add_sync(0xFFFFFFFFu, deg);
-    }
     if (lane == 0 && c_act) {
         atomicAdd(&bctr[0], (unsigned long long)c_act);
         atomicAdd(&bctr[1], c_edges);
@@ -591,12 +638,25 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
+#ifndef NULPA_WARP_ORDER
+#define NULPA_WARP_ORDER 0
+#endif
 constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
+// The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
+// tables (8 KB per warp, p1 = 1023), 4 warps per CTA, 6 CTAs (24 warps) per SM.
+constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
+template <int SLOTS> struct WarpCfg {
+    static constexpr int warps = SLOTS == kWarpSlots ? kWarpWarps : kWideWarps;
+    static constexpr int ctas = SLOTS == kWarpSlots ? kWarpCtasPerSm : kWideCtasPerSm;
+    static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step
+};
 
-template <bool SYNC, bool W, int TIE>
-__global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepArgs a, const VRec *__restrict__ recs,
-                                                                        const unsigned long long *__restrict__ count) {
-    __shared__ __align__(16) uint64_t s_tab[kWarpWarps][kWarpSlots];
+template <bool SYNC, bool W, int TIE, int SLOTS>
+__global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ctas)
+    k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin) {
+    constexpr int kWarpWarps = WarpCfg<SLOTS>::warps;
+    constexpr int U = WarpCfg<SLOTS>::unroll;
+    __shared__ __align__(16) uint64_t s_tab[kWarpWarps][SLOTS];
     __shared__ VRec s_ring[kWarpWarps][2][32];
     __shared__ unsigned long long bctr[2];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -607,12 +667,20 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
     const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
     const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
     const int64_t ng = (nrec + 31) / 32;
+#if NULPA_WARP_ORDER == 1
+    // chunked: warp gw owns groups [gw*G, gw*G + G)
+    const int64_t G = (ng + nw - 1) / nw, g0 = gw * G, gs = 1;
+    const int64_t nq = std::max<int64_t>(0, std::min<int64_t>(G, ng - g0));
+#else
+    // strided: warp gw owns groups gw, gw + nw, ...
+    const int64_t g0 = gw, gs = nw;
     const int64_t nq = gw < ng ? (ng - 1 - gw) / nw + 1 : 0;            // groups of this warp
-    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - (gw + (nq - 1) * nw) * 32) : 0;
+#endif
+    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - (g0 + (nq - 1) * gs) * 32) : 0;
     unsigned long long c_ch = 0, c_che = 0;
     auto grec = [&](int64_t q) -> VRec {                   // lane's record of group q (or empty)
         VRec z{0, 0, 0, 0};
-        const int64_t i = (gw + q * nw) * 32 + lane;
+        const int64_t i = (g0 + q * gs) * 32 + lane;
         return (q < nq && i < nrec) ? recs[i] : z;
     };
     auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
@@ -711,29 +779,33 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
             };
             batch(s0.ka, s0.wa);
             batch(s0.kb, s0.wb);
-            for (uint32_t b = 64; b < dk; b += 64) {
-                const bool u0 = b + lane < dk, u1 = b + 32 + lane < dk;
-                const int32_t i0 = u0 ? __ldcs(pi + b) : -1;
-                const int32_t i1 = u1 ? __ldcs(pi + b + 32) : -1;
-                float x0 = 1.0f, x1 = 1.0f;
-                if (W) {
-                    if (u0) x0 = __ldcs(pw + b);
-                    if (u1) x1 = __ldcs(pw + b + 32);
+            for (uint32_t b = 64; b < dk; b += 32 * U) {
+                // U batches per step: all index loads, then all label gathers in flight
+                int32_t iu[U], qu[U];
+                float xu[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const bool ok = b + 32 * u + lane < dk;
+                    iu[u] = ok ? __ldcs(pi + b + 32 * u) : -1;
+                    xu[u] = 1.0f;
+                    if (W && ok) xu[u] = __ldcs(pw + b + 32 * u);
                 }
-                const int32_t q0 = (i0 >= 0 && i0 != (int32_t)vk) ? a.lab_in[i0] : kEmpty;
-                const int32_t q1 = (i1 >= 0 && i1 != (int32_t)vk) ? a.lab_in[i1] : kEmpty;
-                batch(q0, x0);
-                if (b + 32 < dk) batch(q1, x1);
+#pragma unroll
+                for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != (int32_t)vk) ? a.lab_in[iu[u]] : kEmpty;
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (u == 0 || b + 32 * u < dk) batch(qu[u], xu[u]);
             }
         };
         if (dk <= 32) {
             bool leader;
             const float x = fold(s0.ka, s0.wa, leader);
             if (leader) offer(x, s0.ka);
-        } else if (dk < 64) {
-            table_row(std::integral_constant<uint32_t, 255>());
+        } else if constexpr (SLOTS == kWideSlots) {
+            table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
         } else {
-            table_row(std::integral_constant<uint32_t, 511>());
+            if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
+            else table_row(std::integral_constant<uint32_t, 511>());
         }
         const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
         int32_t cs = kEmpty;
@@ -768,8 +840,8 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
     __syncthreads();
     if (threadIdx.x == 0 && bctr[0]) {
         atomicAdd(&a.ctr[0], bctr[0]);
-        atomicAdd(&a.ctr[9 + 1], bctr[0]);
-        atomicAdd(&a.ctr[13 + 1], bctr[1]);
+        atomicAdd(&a.ctr[9 + bin], bctr[0]);
+        atomicAdd(&a.ctr[13 + bin], bctr[1]);
     }
 }
 
@@ -785,8 +857,8 @@ __global__ void __launch_bounds__(kWarpWarps * 32, kWarpCtasPerSm) k_warp(SweepA
 constexpr int kBlkThreads = 128;
 
 template <bool SYNC, bool W, int TIE>
-__global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_t *__restrict__ list,
-                                                        int64_t n) {
+__global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *__restrict__ recs,
+                                                        const unsigned long long *__restrict__ count) {
     extern __shared__ int32_t dyn[];
     int32_t *Hk = dyn;
     float *Hv = reinterpret_cast<float *>(dyn + kBlockCap);
@@ -796,27 +868,21 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_
     __shared__ int s_changed;
     __shared__ uint32_t s_bw[kBlkThreads / 32], s_rr[kBlkThreads / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    unsigned long long n_act = 0, n_edges = 0, n_changed = 0, n_changed_edges = 0;
+    unsigned long long n_changed = 0, n_changed_edges = 0;
+    const int64_t n = (int64_t)*count;
     const int64_t ngroups = (n + 31) / 32;
     for (int64_t gq = blockIdx.x; gq < ngroups; gq += gridDim.x) {
-        // metadata of 32 consecutive bin entries in one round trip (warp 0)
+        // 32 frontier records (k_frontier: unprocessed vertices, flags already cleared)
         if (wid == 0) {
             const int64_t t = gq * 32 + lane;
-            int f = 0;
             if (t < n) {
-                const int32_t r = list[t];
-                const int64_t v = r + a.row_begin;
-                f = a.flag_in[v];
-                m_r[lane] = r;
-                if (f) {
-                    const int64_t o = a.offsets[r];
-                    m_o[lane] = o;
-                    m_d[lane] = (int32_t)(a.offsets[r + 1] - o);
-                    m_ci[lane] = a.lab_in[v];
-                    if (!SYNC) a.flag_in[v] = 0;           // mark i as processed
-                }
+                const VRec rc = recs[t];
+                m_o[lane] = (int64_t)(((uint64_t)(rc.o_hi_deg & 0xFFFFu) << 32) | rc.o_lo);
+                m_d[lane] = (int32_t)(rc.o_hi_deg >> 16);
+                m_r[lane] = rc.r;
+                m_ci[lane] = rc.ci;
             }
-            const unsigned am = __ballot_sync(0xFFFFFFFFu, f != 0);
+            const unsigned am = __ballot_sync(0xFFFFFFFFu, t < n);
             if (lane == 0) s_act = am;
         }
         __syncthreads();
@@ -899,8 +965,6 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_
                 const int ch = accept_move(cs, m_ci[k], a.pickless);
                 if (ch) a.lab_out[v] = cs;
                 s_changed = ch;
-                n_act += 1;
-                n_edges += deg;
                 n_changed += ch;
                 n_changed_edges += ch ? deg : 0;
             }
@@ -910,14 +974,10 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const int32_
         }
         __syncthreads();
     }
-    if (threadIdx.x == 0 && n_act) {
-        atomicAdd(&a.ctr[1 + 2], n_act);
-        atomicAdd(&a.ctr[5 + 2], n_edges);
-        if (n_changed) {
-            atomicAdd(&a.ctr[0], n_changed);
-            atomicAdd(&a.ctr[9 + 2], n_changed);
-            atomicAdd(&a.ctr[13 + 2], n_changed_edges);
-        }
+    if (threadIdx.x == 0 && n_changed) {
+        atomicAdd(&a.ctr[0], n_changed);
+        atomicAdd(&a.ctr[9 + 2], n_changed);
+        atomicAdd(&a.ctr[13 + 2], n_changed_edges);
     }
 }
 
@@ -1360,6 +1420,7 @@ struct nulpa_graph {
     bool bins_built = false;
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
     void *wrecs = nullptr;          // warp-bin frontier records (VRec [bin_n[1]])
+    void *brecs = nullptr;          // block-bin frontier records (VRec [2 * bin_n[2]]: warp part | CTA part)
     int64_t bin_n[4] = {0, 0, 0, 0};
     int64_t bin_e[4] = {0, 0, 0, 0};
     int64_t bin_maxdeg[4] = {0, 0, 0, 0};
@@ -1405,6 +1466,8 @@ int dalloc(T **p, size_t n) {
 void free_bins(nulpa_graph *g) {
     cudaFree(g->wrecs);
     g->wrecs = nullptr;
+    cudaFree(g->brecs);
+    g->brecs = nullptr;
     for (int b = 0; b < 4; ++b) {
         cudaFree(g->bin_list[b]);
         g->bin_list[b] = nullptr;
@@ -1551,6 +1614,8 @@ int validate_params(const nulpa_params &p) {
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
     if (p.bin_order < 0 || p.bin_order > 2) return fail(NULPA_EINVAL, "bin_order must be 0, 1 or 2");
+    if (p.wide_degree < 1 || p.wide_degree > 512)
+        return fail(NULPA_EINVAL, "wide_degree must be in [1, 512] (wide warp tables hold 1023 slots)");
     if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
         return fail(NULPA_EINVAL, "giant_degree must be in [block_degree, 4096] (CTA tables hold 4095 slots)");
     return NULPA_OK;
@@ -1644,10 +1709,20 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[2];
         CHECK(rec(2, 0));
         if (n > 0) {
+            // frontier split at wide_degree: warp-per-vertex (1023-slot tables) below, CTA-per-vertex above
+            if (!g->brecs) CHECK(dalloc(reinterpret_cast<VRec **>(&g->brecs), (size_t)(2 * n)));
+            VRec *rw = reinterpret_cast<VRec *>(g->brecs), *rb = rw + n;
+            const uint32_t split = (uint32_t)std::max(p.wide_degree, p.block_degree);
+            k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[2], n, 2, rw, ctr + kCtrRecsW,
+                                                                          split, rb, ctr + kCtrRecsB);
+            if (split > (uint32_t)p.block_degree) {
+                k_warp<SYNC, W, TIE, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2);
+                g->stats.launches[2] += 1;
+            }
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, g->bin_list[2], n);
+            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB);
             CU(cudaGetLastError());
-            g->stats.launches[2] += 1;
+            g->stats.launches[2] += 2;
         }
         CHECK(rec(2, 1));
         return NULPA_OK;
@@ -1658,8 +1733,9 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         if (n > 0) {
             if (!g->wrecs) CHECK(dalloc(reinterpret_cast<VRec **>(&g->wrecs), (size_t)n));
             VRec *recs = reinterpret_cast<VRec *>(g->wrecs);
-            k_frontier<SYNC><<<grid_for(n, 256, sms * 8), 256, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs);
-            k_warp<SYNC, W, TIE><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs);
+            k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs,
+                                                                          0xFFFFFFFFu, nullptr, nullptr);
+            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
         }
@@ -1778,6 +1854,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->timing = 0;
     p->tie_rule = NULPA_TIE_SMALLEST;
     p->bin_order = 1;
+    p->wide_degree = 512;
 }
 
 const char *nulpa_last_error(void) { return g_err.c_str(); }

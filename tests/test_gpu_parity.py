@@ -18,14 +18,17 @@ import paper_conf_ipps_sahunk25_b200 as nl
 
 pytestmark = pytest.mark.gpu
 
-# degree-bin configurations: default; every bin populated on small graphs;
-# the paper's two-kernel split (thread < 32 <= block); all-warp; all-block; all-giant
+# degree-bin configurations: default; every bin (and both block-bin kernels)
+# populated on small graphs; the paper's two-kernel split (thread < 32 <=
+# block); all-warp; all-wide-warp (+ CTA kernel for degree >= 512); all-CTA
+# (wide_degree=1); all-giant
 BINS = {
     "default": dict(),
-    "mixed": dict(switch_degree=4, block_degree=12, giant_degree=40),
+    "mixed": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40),
     "paper": dict(switch_degree=32, block_degree=32, giant_degree=4096),
     "warp": dict(switch_degree=1, block_degree=256, giant_degree=4096),
-    "block": dict(switch_degree=1, block_degree=1, giant_degree=4096),
+    "wide": dict(switch_degree=1, block_degree=1, giant_degree=4096),
+    "block": dict(switch_degree=1, block_degree=1, wide_degree=1, giant_degree=4096),
     "giant": dict(switch_degree=1, block_degree=1, giant_degree=1),
 }
 
