@@ -638,8 +638,8 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
-#ifndef NULPA_WARP_ORDER
-#define NULPA_WARP_ORDER 0
+#ifndef NULPA_WARP_BLOCK
+#define NULPA_WARP_BLOCK 1      // record groups per block of the block-cyclic warp schedule
 #endif
 constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
 // The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
@@ -667,20 +667,16 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
     const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
     const int64_t ng = (nrec + 31) / 32;
-#if NULPA_WARP_ORDER == 1
-    // chunked: warp gw owns groups [gw*G, gw*G + G)
-    const int64_t G = (ng + nw - 1) / nw, g0 = gw * G, gs = 1;
-    const int64_t nq = std::max<int64_t>(0, std::min<int64_t>(G, ng - g0));
-#else
-    // strided: warp gw owns groups gw, gw + nw, ...
-    const int64_t g0 = gw, gs = nw;
-    const int64_t nq = gw < ng ? (ng - 1 - gw) / nw + 1 : 0;            // groups of this warp
-#endif
-    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - (g0 + (nq - 1) * gs) * 32) : 0;
+    // block-cyclic: warp gw owns blocks of K consecutive groups: gw, gw + nw, ...
+    constexpr int64_t K = NULPA_WARP_BLOCK;
+    const int64_t NB = ng / K, rem = ng % K;
+    const int64_t nq = (gw < NB ? (NB - 1 - gw) / nw + 1 : 0) * K + ((rem && NB % nw == gw) ? rem : 0);
+    auto gidx = [&](int64_t q) -> int64_t { return ((q / K) * nw + gw) * K + q % K; };
+    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - gidx(nq - 1) * 32) : 0;
     unsigned long long c_ch = 0, c_che = 0;
     auto grec = [&](int64_t q) -> VRec {                   // lane's record of group q (or empty)
         VRec z{0, 0, 0, 0};
-        const int64_t i = (g0 + q * gs) * 32 + lane;
+        const int64_t i = gidx(q) * 32 + lane;
         return (q < nq && i < nrec) ? recs[i] : z;
     };
     auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
