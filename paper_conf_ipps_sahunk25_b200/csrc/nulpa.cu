@@ -15,7 +15,7 @@
 //
 // Kernels of one sweep (lpaMove), launched on the handle's stream, by default
 // in the order thread -> warp -> block -> giant (bin_order 1, hubs last):
-//   k_giant_snapshot / k_giant_accumulate / k_giant_reduce / k_giant_decide / k_giant_mark
+//   k_giant_snapshot / k_giant_accumulate / k_giant_decide / k_giant_finish
 //   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
 //   k_frontier + k_warp   compacted frontier; one warp per vertex, pipelined,
 //                         shared-memory table (<= 511 slots)
@@ -47,8 +47,8 @@ constexpr int kCtrRecsB = 22;            // counter slot: block-bin frontier, CT
 
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
 constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
-constexpr int kGiantChunk = 4096;        // edges per giant chunk
-constexpr int kGiantCap = 8192;          // slots of a chunk table (4096 edges -> p1 = 8191)
+constexpr int kGiantChunk = 2048;        // edges per giant chunk
+constexpr int kGiantCap = 4096;          // slots of a chunk table (2048 edges -> p1 = 4095)
 constexpr int kThreadThreads = 256;
 
 thread_local std::string g_err;
@@ -164,7 +164,7 @@ struct TieOrder {
 // (same slots); R5 linear continuation after kMaxRetries probes.
 // Returns true if the key newly claimed a slot (*slot_out = slot).
 __device__ __forceinline__ bool ht_accumulate(int32_t *Hk, float *Hv, const Hash &h, int32_t k,
-                                              float v, uint32_t *slot_out = nullptr) {
+                                              float v, uint32_t *slot_out = nullptr, float *total_out = nullptr) {
     const uint32_t p1 = h.p1;
     uint32_t i = fastmod((uint32_t)k, h.m1, p1);
     uint32_t di = p1 > 1 ? 1u : 0u;
@@ -176,7 +176,8 @@ __device__ __forceinline__ bool ht_accumulate(int32_t *Hk, float *Hv, const Hash
         if (cur == k || cur == kEmpty) {
             int32_t old = cur == k ? k : atomicCAS(&Hk[i], kEmpty, k);
             if (old == kEmpty || old == k) {
-                atomicAdd(&Hv[i], v);
+                const float prev = atomicAdd(&Hv[i], v);
+                if (total_out) *total_out = __fadd_rn(prev, v);
                 if (slot_out) *slot_out = i;
                 return old == kEmpty;
             }
@@ -192,7 +193,8 @@ __device__ __forceinline__ bool ht_accumulate(int32_t *Hk, float *Hv, const Hash
         if (cur == k || cur == kEmpty) {
             int32_t old = cur == k ? k : atomicCAS(&Hk[i], kEmpty, k);
             if (old == kEmpty || old == k) {
-                atomicAdd(&Hv[i], v);
+                const float prev = atomicAdd(&Hv[i], v);
+                if (total_out) *total_out = __fadd_rn(prev, v);
                 if (slot_out) *slot_out = i;
                 return old == kEmpty;
             }
@@ -273,35 +275,6 @@ __device__ __forceinline__ uint32_t cas_u32(uint32_t addr, uint32_t cmp, uint32_
     uint32_t old;
     asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(addr), "r"(cmp), "r"(val) : "memory");
     return old;
-}
-
-// One 32-edge batch of a warp against a table shared by several warps (the
-// giant chunk tables): lanes holding the same label (match_any) are folded
-// onto their lowest lane (the leader), which claims the label's slot
-// (Algorithm 2 probing, atomicCAS) and adds the group's total with one
-// shared-memory atomicAdd (a CAS loop on this GPU -- there is no native
-// shared float atomicAdd -- contended by at most one lane per warp and
-// label).  Uniform weights: total = count * w.
-template <bool W>
-__device__ __forceinline__ void warp_batch_accumulate_atomic(int32_t *Hk, float *Hv, const Hash &h, int32_t key,
-                                                             float w) {
-    const int lane = threadIdx.x & 31;
-    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
-    const bool leader = key != kEmpty && lane == __ffs(grp) - 1;
-    float sum;
-    if (W) {
-        const unsigned valid = __ballot_sync(0xFFFFFFFFu, key != kEmpty);
-        const float wr = __shfl_sync(0xFFFFFFFFu, w, valid ? __ffs(valid) - 1 : 0);
-        if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == wr)) {
-            sum = (float)__popc(grp) * w;
-        } else {
-            const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-            sum = maxn > 1 ? group_sum(grp, w, maxn) : w;
-        }
-    } else {
-        sum = (float)__popc(grp);
-    }
-    if (leader) atomicAdd(&Hv[ht_claim(Hk, h, key)], sum);
 }
 
 // (weight, tie rank) packed so that an unsigned max gives the largest weight
@@ -649,6 +622,7 @@ template <int SLOTS> struct WarpCfg {
     static constexpr int warps = SLOTS == kWarpSlots ? kWarpWarps : kWideWarps;
     static constexpr int ctas = SLOTS == kWarpSlots ? kWarpCtasPerSm : kWideCtasPerSm;
     static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step
+    static constexpr int block = SLOTS == kWarpSlots ? NULPA_WARP_BLOCK : 1;   // schedule blocks (groups)
 };
 
 template <bool SYNC, bool W, int TIE, int SLOTS>
@@ -667,11 +641,18 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
     const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
     const int64_t ng = (nrec + 31) / 32;
-    // block-cyclic: warp gw owns blocks of K consecutive groups: gw, gw + nw, ...
-    constexpr int64_t K = NULPA_WARP_BLOCK;
-    const int64_t NB = ng / K, rem = ng % K;
-    const int64_t nq = (gw < NB ? (NB - 1 - gw) / nw + 1 : 0) * K + ((rem && NB % nw == gw) ? rem : 0);
-    auto gidx = [&](int64_t q) -> int64_t { return ((q / K) * nw + gw) * K + q % K; };
+    // Balanced block-cyclic schedule: R full rounds in which every warp takes
+    // K consecutive groups (round r, warp gw: groups r*nw*K + gw*K + [0, K)),
+    // then a last round splitting the remaining groups evenly (K2 per warp).
+    // Within its blocks a warp walks consecutive rows in order, so labels
+    // propagate along ID order as in the sequential Algorithm 1 (modularity);
+    // K = 1 is the plain strided schedule.
+    constexpr int64_t K = WarpCfg<SLOTS>::block;
+    const int64_t R = ng / (nw * K), rem = ng - R * nw * K, K2 = (rem + nw - 1) / nw;
+    const int64_t nq = R * K + std::max<int64_t>(0, std::min<int64_t>(K2, rem - gw * K2));
+    auto gidx = [&](int64_t q) -> int64_t {
+        return q < R * K ? (q / K) * nw * K + gw * K + q % K : R * nw * K + gw * K2 + (q - R * K);
+    };
     const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - gidx(nq - 1) * 32) : 0;
     unsigned long long c_ch = 0, c_che = 0;
     auto grec = [&](int64_t q) -> VRec {                   // lane's record of group q (or empty)
@@ -980,10 +961,15 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
 // ---------------------------------------------------------------------------
 // giant vertices (degree >= giant_degree): the row is cut into chunks of
 // kGiantChunk edges, one CTA per chunk.  Each CTA pre-aggregates its chunk in
-// a shared-memory table, then folds the distinct (label, weight) pairs into
-// the vertex's GLOBAL-memory table (p1 = nextPow2(D)-1 slots),
-// recording newly claimed slots in an occupied list so the max-reduce and the
-// clear touch only occupied slots.
+// a shared-memory table (recording the slots it claims), then folds the
+// distinct (label, weight) pairs into the vertex's GLOBAL-memory table
+// (p1 = nextPow2(D)-1 slots) with atomicAdd.  Weights are
+// non-negative (R12), so a label's running totals only grow and the largest
+// total any fold returns is hashtableMaxKey: each CTA folds the best
+// (total, tie rank) it saw into best[gi] with one 64-bit atomicMax -- no
+// scan of the global table.  Newly claimed global slots go to an occupied
+// list, which k_giant_finish clears (and, for moved vertices, the chunk's
+// neighbours are marked there too).
 // ---------------------------------------------------------------------------
 struct GiantArgs {
     const int32_t *verts;        // [ng] local row ids
@@ -1009,14 +995,18 @@ __global__ void k_giant_snapshot(SweepArgs a, GiantArgs g, int64_t ng) {
     g.active[k] = f ? 1 : 0;
     g.changed[k] = 0;
     g.best[k] = 0;
+    g.occ_n[k] = 0;
     if (!SYNC && f) a.flag_in[v] = 0;
 }
 
-template <bool SYNC, bool W>
+template <bool SYNC, bool W, int TIE>
 __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a, GiantArgs g) {
     extern __shared__ int32_t dyn[];
     int32_t *Hk = dyn;
     float *Hv = reinterpret_cast<float *>(dyn + kGiantCap);
+    uint16_t *s_occ = reinterpret_cast<uint16_t *>(dyn + 2 * kGiantCap);   // claimed slots (<= kGiantChunk)
+    __shared__ int s_nocc;
+    __shared__ uint64_t red[kBlockThreads / 32];
     const int64_t c = blockIdx.x;
     const int32_t gi = g.chunk_g[c];
     if (!g.active[gi]) return;
@@ -1027,75 +1017,79 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
         Hk[s] = kEmpty;
         Hv[s] = 0.0f;
     }
+    if (threadIdx.x == 0) s_nocc = 0;
     __syncthreads();
     Hash hc;
     hc.init((uint32_t)(e1 - e0));
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int64_t b = e0 + wid * 32; b < e1; b += kBlockThreads) {
-        int32_t key = kEmpty;
-        float w = 0.0f;
-        if (b + lane < e1) {
-            const int32_t j = __ldcs(a.indices + b + lane);
-            if (j != (int32_t)v) {
-                key = a.lab_in[j];
-                if (W) w = __ldcs(a.weights + b + lane);
+    // two 32-edge batches per warp per step: both index loads, then both gathers in flight
+    for (int64_t b = e0 + wid * 32; b < e1; b += 2 * kBlockThreads) {
+        int32_t key[2] = {kEmpty, kEmpty};
+        float w[2] = {0.0f, 0.0f};
+        int32_t j[2] = {-1, -1};
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const int64_t e = b + u * kBlockThreads + lane;
+            if (e < e1) {
+                j[u] = __ldcs(a.indices + e);
+                if (W) w[u] = __ldcs(a.weights + e);
             }
         }
-        warp_batch_accumulate_atomic<W>(Hk, Hv, hc, key, w);
+#pragma unroll
+        for (int u = 0; u < 2; ++u)
+            if (j[u] >= 0 && j[u] != (int32_t)v) key[u] = a.lab_in[j[u]];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            if (b + u * kBlockThreads >= e1) break;
+            const unsigned grp = __match_any_sync(0xFFFFFFFFu, key[u]);
+            const bool leader = key[u] != kEmpty && lane == __ffs(grp) - 1;
+            float sum;
+            if (W) {
+                const unsigned valid = __ballot_sync(0xFFFFFFFFu, key[u] != kEmpty);
+                const float wr = __shfl_sync(0xFFFFFFFFu, w[u], valid ? __ffs(valid) - 1 : 0);
+                if (__all_sync(0xFFFFFFFFu, key[u] == kEmpty || w[u] == wr)) {
+                    sum = (float)__popc(grp) * w[u];
+                } else {
+                    const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key[u] != kEmpty ? (unsigned)__popc(grp) : 1u);
+                    sum = maxn > 1 ? group_sum(grp, w[u], maxn) : w[u];
+                }
+            } else {
+                sum = (float)__popc(grp);
+            }
+            if (leader) {
+                uint32_t slot;
+                if (ht_accumulate(Hk, Hv, hc, key[u], sum, &slot)) s_occ[atomicAdd(&s_nocc, 1)] = (uint16_t)slot;
+            }
+        }
     }
     __syncthreads();
     Hash hg;
     hg.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
+    TieOrder<TIE> to;
+    to.init(hg);
     int32_t *gk = g.keys + g.table_off[gi];
     float *gv = g.vals + g.table_off[gi];
     int32_t *occ = g.occ + g.table_off[gi];
-    for (uint32_t s = threadIdx.x; s < hc.p1; s += kBlockThreads) {
-        int32_t k = Hk[s];
-        if (k != kEmpty) {
-            uint32_t slot;
-            if (ht_accumulate(gk, gv, hg, k, Hv[s], &slot)) occ[atomicAdd(&g.occ_n[gi], 1)] = (int32_t)slot;
-        }
-    }
-    if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
-}
-
-// hashtableMaxKey for giant vertices, spread over the vertex's chunk CTAs:
-// CTA k of a vertex scans occupied-list entries [k*kGiantChunk, ...), clears
-// those slots, and folds its maximum into best[gi] (global 64-bit atomicMax).
-template <bool SYNC, int TIE>
-__global__ void __launch_bounds__(kBlockThreads) k_giant_reduce(SweepArgs a, GiantArgs g) {
-    const int64_t c = blockIdx.x;
-    const int32_t gi = g.chunk_g[c];
-    if (!g.active[gi]) return;
-    __shared__ uint64_t red[kBlockThreads / 32];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int32_t r = g.verts[gi];
-    const int64_t kc = (g.chunk_e0[c] - a.offsets[r]) / kGiantChunk;
-    int32_t *gk = g.keys + g.table_off[gi];
-    float *gv = g.vals + g.table_off[gi];
-    const int32_t *occ = g.occ + g.table_off[gi];
-    const int64_t cnt = g.occ_n[gi];
-    const int64_t q0 = kc * kGiantChunk, q1 = q0 + kGiantChunk < cnt ? q0 + kGiantChunk : cnt;
-    Hash h;
-    h.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
-    TieOrder<TIE> to;
-    to.init(h);
     uint64_t best = 0;
-    for (int64_t q = q0 + threadIdx.x; q < q1; q += kBlockThreads) {
-        const int32_t sl = occ[q];
-        const uint64_t cd = pack_cand(gv[sl], gk[sl], to);
+    const int nocc = s_nocc;
+    for (int q = threadIdx.x; q < nocc; q += kBlockThreads) {
+        const uint32_t s = s_occ[q];
+        const int32_t k = Hk[s];
+        uint32_t slot;
+        float total;
+        if (ht_accumulate(gk, gv, hg, k, Hv[s], &slot, &total)) occ[atomicAdd(&g.occ_n[gi], 1)] = (int32_t)slot;
+        const uint64_t cd = pack_cand(total, k, to);
         best = cd > best ? cd : best;
-        gk[sl] = kEmpty;
-        gv[sl] = 0.0f;
     }
     best = warp_max_u64(best);
     if (lane == 0) red[wid] = best;
     __syncthreads();
     if (wid == 0) {
-        uint64_t b = lane < kBlockThreads / 32 ? red[lane] : 0;
-        b = warp_max_u64(b);
-        if (lane == 0 && b) atomicMax(&g.best[gi], (unsigned long long)b);
+        uint64_t bb = lane < kBlockThreads / 32 ? red[lane] : 0;
+        bb = warp_max_u64(bb);
+        if (lane == 0 && bb) atomicMax(&g.best[gi], (unsigned long long)bb);
     }
+    if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
 }
 
 // the move rule for every giant vertex (one thread each)
@@ -1103,7 +1097,6 @@ template <bool SYNC, int TIE>
 __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     const int64_t gi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (gi >= ng || !g.active[gi]) return;
-    g.occ_n[gi] = 0;
     const int32_t r = g.verts[gi];
     const int64_t v = r + a.row_begin;
     const int64_t deg = a.offsets[r + 1] - a.offsets[r];
@@ -1124,12 +1117,27 @@ __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     atomicAdd(&a.ctr[1 + 3], 1ull);
 }
 
-__global__ void __launch_bounds__(kBlockThreads) k_giant_mark(SweepArgs a, GiantArgs g) {
+// per chunk CTA: clear its slice of the vertex's occupied list (hashtableClear
+// of the used slots) and, if the vertex moved, mark the chunk's neighbours
+__global__ void __launch_bounds__(kBlockThreads) k_giant_finish(SweepArgs a, GiantArgs g) {
     const int64_t c = blockIdx.x;
     const int32_t gi = g.chunk_g[c];
-    if (!g.changed[gi]) return;
-    for (int64_t e = g.chunk_e0[c] + threadIdx.x; e < g.chunk_e1[c]; e += kBlockThreads)
-        a.flag_out[a.indices[e]] = 1;
+    if (!g.active[gi]) return;
+    const int32_t r = g.verts[gi];
+    const int64_t kc = (g.chunk_e0[c] - a.offsets[r]) / kGiantChunk;
+    int32_t *gk = g.keys + g.table_off[gi];
+    float *gv = g.vals + g.table_off[gi];
+    const int32_t *occ = g.occ + g.table_off[gi];
+    const int64_t cnt = g.occ_n[gi];
+    const int64_t q0 = kc * kGiantChunk, q1 = q0 + kGiantChunk < cnt ? q0 + kGiantChunk : cnt;
+    for (int64_t q = q0 + threadIdx.x; q < q1; q += kBlockThreads) {
+        const int32_t sl = occ[q];
+        gk[sl] = kEmpty;
+        gv[sl] = 0.0f;
+    }
+    if (g.changed[gi])
+        for (int64_t e = g.chunk_e0[c] + threadIdx.x; e < g.chunk_e1[c]; e += kBlockThreads)
+            a.flag_out[a.indices[e]] = 1;
 }
 
 // ---------------------------------------------------------------------------
@@ -1684,19 +1692,18 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             ga.active = g->gactive;
             ga.changed = g->gchanged;
             ga.best = g->gbest;
-            const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float));
+            const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float)) + kGiantChunk * sizeof(uint16_t);
             static bool attr_set = false;   // one per template instantiation
             if (!attr_set) {
-                CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W, TIE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
                 attr_set = true;
             }
             k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, cs>>>(a, ga, ng);
-            k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
-            k_giant_reduce<SYNC, TIE><<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
+            k_giant_accumulate<SYNC, W, TIE><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
             k_giant_decide<SYNC, TIE><<<grid_for(ng, 128), 128, 0, cs>>>(a, ga, ng);
-            k_giant_mark<<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
+            k_giant_finish<<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
             CU(cudaGetLastError());
-            g->stats.launches[3] += 5;
+            g->stats.launches[3] += 4;
         }
         CHECK(rec(3, 1));
         return NULPA_OK;
