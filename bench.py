@@ -48,6 +48,10 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=6_000_000, help="vertices of the oracle's web-graph sample")
     ap.add_argument("--extra", action="store_true", help="also time the unit-weight fast path and sync mode")
+    ap.add_argument("--param", action="append", default=[], metavar="KEY=INT",
+                    help="override an nulpa_params field (experiments), e.g. --param first_sweep_block=1")
+    ap.add_argument("--quality-runs", type=int, default=4,
+                    help="extra untimed runs whose modularity is reported next to the timed run's")
     return ap.parse_args()
 
 
@@ -237,6 +241,9 @@ def run_ours(args):
     stream = torch.cuda.current_stream()
     gg = nl.Graph(g.offsets, g.indices, weights)
     params = dict(timing=1)
+    for kv in args.param:
+        k, v = kv.split("=")
+        params[k] = int(v)
     for _ in range(args.warmup):
         gg.run(**params)
     torch.cuda.synchronize()
@@ -254,6 +261,10 @@ def run_ours(args):
     ms = ev0.elapsed_time(ev1) / args.steps
     value = M / (ms / 1e3)
     q = gg.modularity()
+    q_runs = [q]
+    for _ in range(args.quality_runs):      # asynchronous LPA's result depends on the schedule
+        gg.run(**params)
+        q_runs.append(gg.modularity())
     launches = sum(sum(s["launches"]) + s["other_launches"] for s in stats)
 
     # roofline of the dominant kernel (bin with the largest summed kernel time)
@@ -289,10 +300,11 @@ def run_ours(args):
             "config": {"workload": args.config, "N": N, "M": M, "weights": args.weights,
                        "generator_seconds": round(t_gen, 1), "scale": args.scale,
                        "l2": f"inputs ({(M * (8 if weighted else 4) + 8 * N) / 1e9:.1f} GB) larger than the 126 MB L2; no flush",
-                       "params": {"tolerance": 0.05, "max_iterations": 20, "pickless_period": 4, "mode": "async"},
+                       "params": {"tolerance": 0.05, "max_iterations": 20, "pickless_period": 4, "mode": "async",
+                                  **{k: v for k, v in params.items() if k != "timing"}},
                        "parallelism": "single GPU"},
             "iterations": st0["iterations"], "converged": st0["converged"], "changed": st0["changed"],
-            "modularity": q,
+            "modularity": q, "modularity_runs": [round(x, 4) for x in q_runs],
             "bins": {BINS[b]: {"vertices": st0["bin_vertices"][b], "edges": st0["bin_edges"][b],
                                "kernel_ms_per_run": round(tot_ms[b] / args.steps, 3)} for b in range(4)},
             "roofline": roof, "gpu_launches": launches, "clocks": ck,

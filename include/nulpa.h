@@ -77,6 +77,13 @@ typedef struct nulpa_params {
                                     <= 1/2); degree >= this -> one CTA per vertex.  Range
                                     [1, 512]; <= block_degree sends the whole bin to the CTA
                                     kernel.  B200 default 512                                   */
+    int32_t first_sweep_block;   /* warp-bin schedule of the first sweep after a reset: each warp
+                                    walks blocks of this many consecutive 32-vertex record groups
+                                    (balanced block-cyclic; 1 = strided).  Larger blocks let labels
+                                    propagate along ID order within a warp as in the sequential
+                                    Algorithm 1 (better modularity) at some memory-latency cost.
+                                    Range [1, 1024]; default 64     */
+    int32_t sweep_block;         /* the same for every later sweep; default 1                   */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0

@@ -52,6 +52,8 @@ class Params(ctypes.Structure):
         ("tie_rule", ctypes.c_int32),
         ("bin_order", ctypes.c_int32),
         ("wide_degree", ctypes.c_int32),
+        ("first_sweep_block", ctypes.c_int32),
+        ("sweep_block", ctypes.c_int32),
     ]
 
 

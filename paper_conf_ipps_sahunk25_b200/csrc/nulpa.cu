@@ -315,6 +315,7 @@ struct SweepArgs {
     uint8_t *flag_out;
     int64_t row_begin;
     int pickless;
+    int sched_block;           // warp-bin schedule: record groups per block (k_warp)
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 
@@ -611,9 +612,7 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
-#ifndef NULPA_WARP_BLOCK
-#define NULPA_WARP_BLOCK 1      // record groups per block of the block-cyclic warp schedule
-#endif
+
 constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
 // The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
 // tables (8 KB per warp, p1 = 1023), 4 warps per CTA, 6 CTAs (24 warps) per SM.
@@ -622,7 +621,6 @@ template <int SLOTS> struct WarpCfg {
     static constexpr int warps = SLOTS == kWarpSlots ? kWarpWarps : kWideWarps;
     static constexpr int ctas = SLOTS == kWarpSlots ? kWarpCtasPerSm : kWideCtasPerSm;
     static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step
-    static constexpr int block = SLOTS == kWarpSlots ? NULPA_WARP_BLOCK : 1;   // schedule blocks (groups)
 };
 
 template <bool SYNC, bool W, int TIE, int SLOTS>
@@ -647,7 +645,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     // Within its blocks a warp walks consecutive rows in order, so labels
     // propagate along ID order as in the sequential Algorithm 1 (modularity);
     // K = 1 is the plain strided schedule.
-    constexpr int64_t K = WarpCfg<SLOTS>::block;
+    const int64_t K = SLOTS == kWarpSlots ? a.sched_block : 1;
     const int64_t R = ng / (nw * K), rem = ng - R * nw * K, K2 = (rem + nw - 1) / nw;
     const int64_t nq = R * K + std::max<int64_t>(0, std::min<int64_t>(K2, rem - gw * K2));
     auto gidx = [&](int64_t q) -> int64_t {
@@ -1440,6 +1438,7 @@ struct nulpa_graph {
     unsigned long long *ctr = nullptr;       // device [kMaxIter+1][kCtr]
     unsigned long long *ctr_host = nullptr;  // pinned
     int sweep_slot = 0;                      // counter slot used by nulpa_sweep
+    int64_t sweeps_since_reset = 0;          // selects first_sweep_block vs sweep_block
     // modularity scratch
     double *Sigma = nullptr;
     double *macc = nullptr;
@@ -1618,6 +1617,8 @@ int validate_params(const nulpa_params &p) {
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
     if (p.bin_order < 0 || p.bin_order > 2) return fail(NULPA_EINVAL, "bin_order must be 0, 1 or 2");
+    if (p.first_sweep_block < 1 || p.first_sweep_block > 1024 || p.sweep_block < 1 || p.sweep_block > 1024)
+        return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [1, 1024]");
     if (p.wide_degree < 1 || p.wide_degree > 512)
         return fail(NULPA_EINVAL, "wide_degree must be in [1, 512] (wide warp tables hold 1023 slots)");
     if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
@@ -1655,6 +1656,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     a.weights = g->weights;
     a.row_begin = g->row_begin;
     a.pickless = pickless;
+    a.sched_block = g->sweeps_since_reset == 0 ? p.first_sweep_block : p.sweep_block;
     a.ctr = ctr;
     if (SYNC) {
         CU(cudaMemcpyAsync(g->labels_prev, g->labels, g->n_global * sizeof(int32_t), cudaMemcpyDeviceToDevice, g->stream));
@@ -1794,22 +1796,26 @@ int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long lon
         CHECK(dalloc(&g->flags_prev, (size_t)g->n_global));
     }
     const int sel = (p.mode == NULPA_SYNC ? 4 : 0) + (w ? 2 : 0) + (p.tie_rule ? 1 : 0);
+    int r;
     switch (sel) {
-    case 0: return sweep_impl<false, false, 0>(g, pickless, p, ctr, timing, slot);
-    case 1: return sweep_impl<false, false, 1>(g, pickless, p, ctr, timing, slot);
-    case 2: return sweep_impl<false, true, 0>(g, pickless, p, ctr, timing, slot);
-    case 3: return sweep_impl<false, true, 1>(g, pickless, p, ctr, timing, slot);
-    case 4: return sweep_impl<true, false, 0>(g, pickless, p, ctr, timing, slot);
-    case 5: return sweep_impl<true, false, 1>(g, pickless, p, ctr, timing, slot);
-    case 6: return sweep_impl<true, true, 0>(g, pickless, p, ctr, timing, slot);
-    default: return sweep_impl<true, true, 1>(g, pickless, p, ctr, timing, slot);
+    case 0: r = sweep_impl<false, false, 0>(g, pickless, p, ctr, timing, slot); break;
+    case 1: r = sweep_impl<false, false, 1>(g, pickless, p, ctr, timing, slot); break;
+    case 2: r = sweep_impl<false, true, 0>(g, pickless, p, ctr, timing, slot); break;
+    case 3: r = sweep_impl<false, true, 1>(g, pickless, p, ctr, timing, slot); break;
+    case 4: r = sweep_impl<true, false, 0>(g, pickless, p, ctr, timing, slot); break;
+    case 5: r = sweep_impl<true, false, 1>(g, pickless, p, ctr, timing, slot); break;
+    case 6: r = sweep_impl<true, true, 0>(g, pickless, p, ctr, timing, slot); break;
+    default: r = sweep_impl<true, true, 1>(g, pickless, p, ctr, timing, slot); break;
     }
+    ++g->sweeps_since_reset;
+    return r;
 }
 
 int reset_state(nulpa_graph *g) {
     k_init_state<<<grid_for(g->n_global, 256, num_sms() * 16), 256, 0, g->stream>>>(g->labels, g->flags, g->n_global);
     CU(cudaGetLastError());
     g->stats.other_launches += 1;
+    g->sweeps_since_reset = 0;
     return NULPA_OK;
 }
 
@@ -1858,6 +1864,8 @@ void nulpa_default_params(nulpa_params *p) {
     p->tie_rule = NULPA_TIE_SMALLEST;
     p->bin_order = 1;
     p->wide_degree = 512;
+    p->first_sweep_block = 64;
+    p->sweep_block = 1;
 }
 
 const char *nulpa_last_error(void) { return g_err.c_str(); }

@@ -48,7 +48,7 @@ def test_struct_layout_matches_header(lib):
     assert p.tolerance == 0.05 and p.max_iterations == 20 and p.pickless_period == 4
     assert p.mode == nl.ASYNC and p.reset == 1
     assert 1 <= p.switch_degree <= p.block_degree <= p.giant_degree
-    assert ctypes.sizeof(nl.Params) == 8 + 11 * 4 + 4   # 11 int32 fields, padded to 8
+    assert ctypes.sizeof(nl.Params) == 8 + 13 * 4 + 4   # 13 int32 fields, padded to 8
     assert 1 <= p.wide_degree <= 512
     assert nl.nulpa_version().startswith("nulpa")
 
