@@ -17,9 +17,11 @@ for r in rows[hi + 1:]:
     name[r[iid]] = r[ik]
 def dram(k):
     return per[k]["dram__bytes_read.sum"] + per[k]["dram__bytes_write.sum"]
-warp = [k for k in per if "k_warp" in name[k]]
-front = [k for k in per if "k_frontier" in name[k]]
-assert len(warp) == len(front), (len(warp), len(front))
+ids = sorted(per, key=int)
+# the warp bin of a sweep = the k_frontier launch right before each k_warp<..., 512> launch
+warp = [k for k in ids if "k_warp" in name[k] and "512>" in name[k]]
+front = [ids[ids.index(k) - 1] for k in warp]
+assert all("k_frontier" in name[f] for f in front)
 b = [dram(f) + dram(w) for f, w in zip(front, warp)]
 out = {"workload": workload, "weights": weights, "bin": "warp", "kernels": ["k_frontier", "k_warp"],
        "sweeps": len(b), "dram_bytes_per_sweep": sum(b) / len(b), "per_sweep": b,
