@@ -82,7 +82,7 @@ typedef struct nulpa_params {
                                     (balanced block-cyclic; 1 = strided).  Larger blocks let labels
                                     propagate along ID order within a warp as in the sequential
                                     Algorithm 1 (better modularity) at some memory-latency cost.
-                                    Range [1, 1024]; default 64     */
+                                    Range [1, 1024]; default 128    */
     int32_t sweep_block;         /* the same for every later sweep; default 1                   */
 } nulpa_params;
 
