@@ -300,8 +300,7 @@ def run_ours(args):
             "config": {"workload": args.config, "N": N, "M": M, "weights": args.weights,
                        "generator_seconds": round(t_gen, 1), "scale": args.scale,
                        "l2": f"inputs ({(M * (8 if weighted else 4) + 8 * N) / 1e9:.1f} GB) larger than the 126 MB L2; no flush",
-                       "params": {"tolerance": 0.05, "max_iterations": 20, "pickless_period": 4, "mode": "async",
-                                  **{k: v for k, v in params.items() if k != "timing"}},
+                       "params": effective_params(params),
                        "parallelism": "single GPU"},
             "iterations": st0["iterations"], "converged": st0["converged"], "changed": st0["changed"],
             "modularity": q, "modularity_runs": [round(x, 4) for x in q_runs],
@@ -412,6 +411,15 @@ def run_distributed(args, rank, world, local):
     dist.barrier()
     dist.destroy_process_group()
     return 0
+
+
+def effective_params(overrides) -> dict:
+    """The nulpa_params the timed runs used (library defaults + --param overrides)."""
+    import paper_conf_ipps_sahunk25_b200 as nl
+    p = nl.nulpa_default_params(**{k: v for k, v in overrides.items() if k != "timing"})
+    d = {name: getattr(p, name) for name, _ in p._fields_ if name not in ("timing", "reset")}
+    d["mode"] = "async" if d["mode"] == nl.ASYNC else "sync"
+    return d
 
 
 def main():
