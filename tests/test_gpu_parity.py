@@ -25,7 +25,7 @@ pytestmark = pytest.mark.gpu
 BINS = {
     "default": dict(),
     "mixed": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40),
-    "paper": dict(switch_degree=32, block_degree=32, giant_degree=4096),
+    "paper": dict(switch_degree=32, block_degree=32, wide_degree=1, giant_degree=4096),
     "warp": dict(switch_degree=1, block_degree=256, giant_degree=4096),
     "wide": dict(switch_degree=1, block_degree=1, giant_degree=4096),
     "block": dict(switch_degree=1, block_degree=1, wide_degree=1, giant_degree=4096),
@@ -298,6 +298,58 @@ def test_invalid_params_raise():
         gg.run(block_degree=300)
     with pytest.raises(nl.NulpaError):
         gg.run(max_iterations=100)
+    with pytest.raises(nl.NulpaError):
+        gg.run(wide_degree=513)
+    with pytest.raises(nl.NulpaError):
+        gg.run(first_sweep_block=0)
+    with pytest.raises(nl.NulpaError):
+        gg.run(sweep_block=2000)
+
+
+# warp-bin schedules: (first_sweep_block, sweep_block); 3 and 5 leave ragged
+# last rounds on every test graph
+SCHEDULES = [(1, 1), (3, 5), (128, 1), (1024, 1024)]
+
+
+@pytest.mark.parametrize("gname", ["sbm", "web", "rmat", "kmer"])
+@pytest.mark.parametrize("sched", SCHEDULES)
+def test_sync_schedule_independent(gname, sched):
+    """A synchronous (Jacobi) run reads only the previous sweep's labels, so
+    the warp schedule must not change a single label: bit-exact against the
+    oracle for every schedule (also checks that the block-cyclic schedule
+    visits every frontier record exactly once)."""
+    g = GRAPHS[gname](False)
+    C, it, dn = oracle.lpa(host(g), sync=True)
+    gg = to_gpu(g)
+    st = gg.run(mode=nl.SYNC, first_sweep_block=sched[0], sweep_block=sched[1], switch_degree=1)
+    assert st["iterations"] == it and st["changed"] == list(dn)
+    np.testing.assert_array_equal(gg.labels(device=False).numpy(), C)
+
+
+@pytest.mark.parametrize("gname", ["sbm", "web", "road", "kmer"])
+@pytest.mark.parametrize("sched", SCHEDULES)
+def test_async_schedule_invariants_and_quality(gname, sched):
+    """Asynchronous runs under every schedule: dN = changed labels, labels
+    from own/neighbour labels, Pick-Less never increases a label, and
+    modularity within 0.02 of the lower of the oracle's two schedules."""
+    g = GRAPHS[gname](False)
+    h = host(g)
+    gg = to_gpu(g)
+    gg.reset()
+    C = gg.labels(device=False).numpy()
+    kw = dict(first_sweep_block=sched[0], sweep_block=sched[1])
+    for l in range(6):
+        pl = l % 4 == 0
+        dn = gg.sweep(pl, mode=nl.ASYNC, **kw)
+        C2 = gg.labels(device=False).numpy()
+        assert dn == int((C2 != C).sum())
+        check_async_sweep(h, C, C2, pl)
+        C = C2
+    C_o, _, _ = oracle.lpa(h)
+    C_s, _, _ = oracle.lpa(h, sync=True)
+    q_o = min(oracle.modularity(h, C_o), oracle.modularity(h, C_s))
+    gg.run(**kw)
+    assert oracle.modularity(h, gg.labels(device=False).numpy()) >= q_o - 0.02
 
 
 # ---------------------------------------------------------------------------
