@@ -346,21 +346,26 @@ def e2e(args, g, weights, gg_dev):
     h2d = off_h.numel() * 8 + idx_h.numel() * 4 + (0 if w_h is None else w_h.numel() * 4)
     d2h = lab_h.numel() * 4
     steps = max(1, min(args.steps, 3))
-    times = []
+    times, parts = [], []
     for it in range(steps + 1):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        h = nl.nulpa_create(off_h, idx_h, w_h)
+        h = nl.nulpa_create(off_h, idx_h, w_h)        # cudaMalloc + H2D copy + degree bins
+        ta = time.perf_counter()
         nl.nulpa_run(h, nl.nulpa_default_params())
+        tb = time.perf_counter()
         nl.nulpa_labels(h, lab_h)
         torch.cuda.synchronize()
         t1 = time.perf_counter()
         nl.nulpa_destroy(h)
         if it > 0:            # first one warms the allocator
             times.append(t1 - t0)
+            parts.append((ta - t0, tb - ta, t1 - tb))
     sec = sum(times) / len(times)
+    avg = [sum(p[k] for p in parts) / len(parts) * 1e3 for k in range(3)]
     return {"value": g.M / sec, "unit": "edges/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-            "ms_per_step": sec * 1e3, "steps": len(times)}
+            "ms_per_step": sec * 1e3, "steps": len(times),
+            "ms_breakdown": {"create_h2d": round(avg[0], 1), "run": round(avg[1], 1), "labels_d2h": round(avg[2], 1)}}
 
 
 def run_distributed(args, rank, world, local):
