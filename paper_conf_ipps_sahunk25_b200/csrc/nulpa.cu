@@ -43,6 +43,8 @@ constexpr int kCtr = 24;                 // counters per iteration
 constexpr int kCtrRecs = 20;             // counter slot: warp-bin frontier size
 constexpr int kCtrRecsW = 21;            // counter slot: block-bin frontier, warp-per-vertex part
 constexpr int kCtrRecsB = 22;            // counter slot: block-bin frontier, CTA-per-vertex part
+constexpr int kCtrSchedW = 17;           // counter slot: dynamic schedule of the warp-bin k_warp
+constexpr int kCtrSchedB = 18;           // counter slot: dynamic schedule of the wide k_warp
 // counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
 
 constexpr int kBlockThreads = 512;       // k_block / giant kernels
@@ -612,6 +614,12 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
+#ifndef NULPA_GUIDED_C
+#define NULPA_GUIDED_C 1                 // guided chunk = min(K, groups left / (C * warps)) ...
+#endif
+#ifndef NULPA_GUIDED_MIN
+#define NULPA_GUIDED_MIN 1               // ... but at least min(K, this)
+#endif
 
 constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
 // The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
@@ -625,7 +633,8 @@ template <int SLOTS> struct WarpCfg {
 
 template <bool SYNC, bool W, int TIE, int SLOTS>
 __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ctas)
-    k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin) {
+    k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin,
+           unsigned long long *sched) {
     constexpr int kWarpWarps = WarpCfg<SLOTS>::warps;
     constexpr int U = WarpCfg<SLOTS>::unroll;
     __shared__ __align__(16) uint64_t s_tab[kWarpWarps][SLOTS];
@@ -651,19 +660,38 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     auto gidx = [&](int64_t q) -> int64_t {
         return q < R * K ? (q / K) * nw * K + gw * K + q % K : R * nw * K + gw * K2 + (q - R * K);
     };
-    const int64_t nv = nq ? (nq - 1) * 32 + std::min<int64_t>(32, nrec - gidx(nq - 1) * 32) : 0;
+    // K > 1: dynamic (guided) chunks instead -- a warp grabs its next chunk of
+    // min(K, groups left / nw) groups from a global counter.  A static K-block
+    // schedule gives each warp only ~2 blocks per sweep (a block of 128 groups
+    // is ~1/2 of a warp's sweep), so unequal block weights left a long tail
+    // (sweep 0: 26 ms vs 20 ms strided); guided chunks shrink toward the end.
+    const bool dyn = K > 1;
+    int64_t cur = 0, lim = dyn ? 0 : nq;                   // static: group counter q < nq; dynamic: chunk [cur, lim)
     unsigned long long c_ch = 0, c_che = 0;
-    auto grec = [&](int64_t q) -> VRec {                   // lane's record of group q (or empty)
+    auto grec_next = [&]() -> VRec {                       // lane's record of the warp's next group (or empty)
         VRec z{0, 0, 0, 0};
-        const int64_t i = gidx(q) * 32 + lane;
-        return (q < nq && i < nrec) ? recs[i] : z;
+        if (dyn && cur >= lim) {
+            unsigned long long start = 0, size = 1;
+            if (lane == 0) {
+                const int64_t left = ng - (int64_t)*(volatile unsigned long long *)sched;
+                size = (unsigned long long)std::max<int64_t>(std::min<int64_t>(K, NULPA_GUIDED_MIN),
+                                                             std::min<int64_t>(K, left / (NULPA_GUIDED_C * nw)));
+                start = atomicAdd(sched, size);
+            }
+            cur = (int64_t)__shfl_sync(0xFFFFFFFFu, start, 0);
+            lim = std::min<int64_t>(ng, cur + (int64_t)__shfl_sync(0xFFFFFFFFu, size, 0));
+        }
+        if (cur >= lim) return z;
+        const int64_t i = (dyn ? cur : gidx(cur)) * 32 + lane;
+        ++cur;
+        return i < nrec ? recs[i] : z;
     };
     auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
     auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
-    s_ring[wid][0][lane] = grec(0);                      // zero records (degree 0) past the end
-    s_ring[wid][1][lane] = grec(1);
-    VRec pend = grec(2);
+    s_ring[wid][0][lane] = grec_next();                  // zero records (degree 0) past the end
+    s_ring[wid][1][lane] = grec_next();
+    VRec pend = grec_next();
     __syncwarp();
     // pipeline registers of one vertex: entries lane and lane+32 of its row
     // (index j, weight w, neighbour label k)
@@ -705,7 +733,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         if ((n & 31) == 0 && n > 0) {
             // entering group q = n/32: group q+1 goes where group q-1 was, group q+2 is requested
             s_ring[wid][((n >> 5) + 1) & 1][lane] = pend;
-            pend = grec((n >> 5) + 2);
+            pend = grec_next();
             __syncwarp();
         }
         load_row(n + 2, s2.ja, s2.jb, s2.wa, s2.wb);
@@ -803,7 +831,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         }
     };
     // (unrolling by 3 so the stages rotate by renaming overflows the instruction cache: 30% slower)
-    for (int n = 0; n < (int)nv; ++n) {
+    for (int n = 0; r_d(rrec(n)) != 0; ++n) {           // records have degree >= 1; zero record = end
         step(n, SA, SB, SC);
         SA = SB;
         SB = SC;
@@ -1721,7 +1749,8 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[2], n, 2, rw, ctr + kCtrRecsW,
                                                                           split, rb, ctr + kCtrRecsB);
             if (split > (uint32_t)p.block_degree) {
-                k_warp<SYNC, W, TIE, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2);
+                k_warp<SYNC, W, TIE, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2,
+                                                                                               ctr + kCtrSchedB);
                 g->stats.launches[2] += 1;
             }
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
@@ -1740,7 +1769,8 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             VRec *recs = reinterpret_cast<VRec *>(g->wrecs);
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs,
                                                                           0xFFFFFFFFu, nullptr, nullptr);
-            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1);
+            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
+                                                                                          ctr + kCtrSchedW);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
         }

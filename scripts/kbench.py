@@ -12,7 +12,9 @@ ap.add_argument("--weights", default="ones")
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--async-too", action="store_true")
 ap.add_argument("--capture", default="", help="A or B: one synchronous sweep inside cudaProfilerStart/Stop (ncu --profile-from-start off)")
+ap.add_argument("--param", action="append", default=[], metavar="KEY=INT", help="nulpa_params override for the timed sweeps")
 a = ap.parse_args()
+P = {kv.split("=")[0]: int(kv.split("=")[1]) for kv in a.param}
 g = synth.make(a.config, device="cuda")
 w = torch.ones(g.M, dtype=torch.float32, device="cuda") if a.weights == "ones" else None
 gg = nl.Graph(g.offsets, g.indices, w)
@@ -27,7 +29,7 @@ if a.capture:
     gg.set_labels(L, ones)
     torch.cuda.synchronize()
     torch.cuda.profiler.start()
-    gg.sweep(a.capture == "A", mode=nl.SYNC)
+    gg.sweep(a.capture == "A", mode=nl.SYNC, **P)
     torch.cuda.synchronize()
     torch.cuda.profiler.stop()
     sys.exit(0)
@@ -39,7 +41,7 @@ for name, L in (("A:init", Linit), ("B:converged", Lconv)):
             gg.set_labels(L, ones)
             torch.cuda.synchronize()
             e0.record()
-            gg.sweep(name.startswith("A"), mode=mode)
+            gg.sweep(name.startswith("A"), mode=mode, **P)
             e1.record()
             torch.cuda.synchronize()
             ts.append(e0.elapsed_time(e1))
