@@ -1895,7 +1895,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->bin_order = 1;
     p->wide_degree = 512;
     p->first_sweep_block = 128;
-    p->sweep_block = 1;
+    p->sweep_block = 4;
 }
 
 const char *nulpa_last_error(void) { return g_err.c_str(); }
