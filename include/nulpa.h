@@ -71,7 +71,9 @@ typedef struct nulpa_params {
     int32_t bin_order;           /* 1 (default): thread, warp, block, giant bins in that order
                                     within a sweep (hubs last); 0: giant, block, warp, thread;
                                     2: block + giant on a second stream, concurrent with
-                                    thread + warp                                               */
+                                    thread + warp; 3: warp bin on a high-priority stream, block
+                                    + giant on a low-priority stream released after the
+                                    warp-bin frontier (they fill the warp bin's tail; +1%)      */
     int32_t wide_degree;         /* within the block bin: degree < this -> one warp per vertex
                                     with a warp-private 1023-slot shared-memory table (load
                                     <= 1/2); degree >= this -> one CTA per vertex.  Range

@@ -1478,6 +1478,8 @@ struct nulpa_graph {
     bool events = false;
     cudaStream_t side = nullptr;             // bin_order 2: block + giant bins
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaStream_t hi = nullptr;               // bin_order 3: high-priority stream for the warp bin
+    cudaEvent_t ev_mid = nullptr, ev_join2 = nullptr;
     nulpa_stats stats;
 };
 
@@ -1644,7 +1646,7 @@ int validate_params(const nulpa_params &p) {
     if (p.block_degree < p.switch_degree || p.block_degree > 256)
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
-    if (p.bin_order < 0 || p.bin_order > 2) return fail(NULPA_EINVAL, "bin_order must be 0, 1 or 2");
+    if (p.bin_order < 0 || p.bin_order > 3) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2 or 3");
     if (p.first_sweep_block < 1 || p.first_sweep_block > 1024 || p.sweep_block < 1 || p.sweep_block > 1024)
         return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [1, 1024]");
     if (p.wide_degree < 1 || p.wide_degree > 512)
@@ -1761,6 +1763,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(2, 1));
         return NULPA_OK;
     };
+    bool mid_fork = false;                        // bin_order 3: record ev_mid after the warp-bin frontier
     auto run_warp = [&]() -> int {
         const int64_t n = g->bin_n[1];
         CHECK(rec(1, 0));
@@ -1769,6 +1772,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             VRec *recs = reinterpret_cast<VRec *>(g->wrecs);
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs,
                                                                           0xFFFFFFFFu, nullptr, nullptr);
+            if (mid_fork) CU(cudaEventRecord(g->ev_mid, cs));
             k_warp<SYNC, W, TIE, kWarpSlots><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
                                                                                           ctr + kCtrSchedW);
             CU(cudaGetLastError());
@@ -1792,6 +1796,39 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(run_block());
         CHECK(run_warp());
         CHECK(run_thread());
+    } else if (p.bin_order == 3) {
+        // thread bin on the caller's stream; warp bin on a high-priority
+        // stream; block + giant bins on a low-priority side stream released
+        // after the warp-bin frontier: k_warp's CTAs take every SM's register
+        // file first, the side kernels' CTAs fill SMs as warp-bin CTAs retire
+        // (the warp bin's tail) -- asynchronous reads of concurrently written
+        // labels are what the asynchronous sweep already does
+        if (!g->hi) {
+            int least = 0, greatest = 0;
+            CU(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+            CU(cudaStreamCreateWithPriority(&g->hi, cudaStreamNonBlocking, greatest));
+            if (!g->side) CU(cudaStreamCreateWithPriority(&g->side, cudaStreamNonBlocking, least));
+            if (!g->ev_fork) CU(cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming));
+            if (!g->ev_join) CU(cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming));
+            CU(cudaEventCreateWithFlags(&g->ev_mid, cudaEventDisableTiming));
+            CU(cudaEventCreateWithFlags(&g->ev_join2, cudaEventDisableTiming));
+        }
+        CHECK(run_thread());
+        CU(cudaEventRecord(g->ev_fork, g->stream));
+        CU(cudaStreamWaitEvent(g->hi, g->ev_fork, 0));
+        CU(cudaEventRecord(g->ev_mid, g->hi));          // (re-recorded after the frontier if the bin is non-empty)
+        cs = g->hi;
+        mid_fork = true;
+        CHECK(run_warp());
+        CU(cudaEventRecord(g->ev_join, g->hi));
+        CU(cudaStreamWaitEvent(g->side, g->ev_mid, 0));
+        cs = g->side;
+        CHECK(run_block());
+        CHECK(run_giant());
+        CU(cudaEventRecord(g->ev_join2, g->side));
+        cs = g->stream;
+        CU(cudaStreamWaitEvent(g->stream, g->ev_join, 0));
+        CU(cudaStreamWaitEvent(g->stream, g->ev_join2, 0));
     } else if (p.bin_order == 2) {
         // block + giant bins on a side stream, concurrent with thread + warp:
         // their latency-bound CTAs fill the SMs the warp bin leaves idle
@@ -2197,6 +2234,12 @@ int nulpa_destroy(nulpa_graph *g) {
     cudaFree(g->Sigma);
     cudaFree(g->macc);
     cudaFree(g->Kdeg);
+    if (g->hi) {
+        cudaStreamSynchronize(g->hi);
+        cudaStreamDestroy(g->hi);
+        cudaEventDestroy(g->ev_mid);
+        cudaEventDestroy(g->ev_join2);
+    }
     if (g->side) {
         cudaStreamSynchronize(g->side);
         cudaStreamDestroy(g->side);

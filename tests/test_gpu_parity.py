@@ -30,6 +30,7 @@ BINS = {
     "wide": dict(switch_degree=1, block_degree=1, giant_degree=4096),
     "block": dict(switch_degree=1, block_degree=1, wide_degree=1, giant_degree=4096),
     "giant": dict(switch_degree=1, block_degree=1, giant_degree=1),
+    "concurrent": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40, bin_order=3),
 }
 
 
@@ -165,7 +166,7 @@ def check_async_sweep(h, C_before, C_after, pickless):
 
 
 @pytest.mark.parametrize("gname", ["sbm", "web", "hub", "rmat", "road", "kmer", "karate", "cliques"])
-@pytest.mark.parametrize("bins", ["default", "mixed"])
+@pytest.mark.parametrize("bins", ["default", "mixed", "concurrent"])
 def test_async_sweep_invariants(gname, bins):
     g = GRAPHS[gname](False)
     h = host(g)
