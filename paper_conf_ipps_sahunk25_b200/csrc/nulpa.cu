@@ -1501,38 +1501,74 @@ struct nulpa_graph {
 
 namespace {
 
+// Device memory of every handle comes from one stream-ordered memory pool per
+// device that keeps up to kPoolKeep bytes after they are freed: creating and
+// destroying handles of the same size (the end-to-end path creates one per
+// call) then reuses mapped memory instead of paying cudaMalloc / cudaFree of
+// ~18 GB each time (measured 13-400 ms per call, varying).  Allocations are
+// made on the legacy stream and synchronised before use on any stream; frees
+// happen only after the handle's stream is idle.
+constexpr uint64_t kPoolKeep = UINT64_C(48) << 30;
+cudaMemPool_t device_pool() {
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) return nullptr;
+    if (!pools[dev]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        if (cudaMemPoolCreate(&pools[dev], &props) != cudaSuccess) {
+            pools[dev] = nullptr;
+            return nullptr;
+        }
+        uint64_t keep = kPoolKeep;
+        cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    return pools[dev];
+}
+
 template <typename T>
 int dalloc(T **p, size_t n) {
     if (n == 0) n = 1;
-    cudaError_t e = cudaMalloc((void **)p, n * sizeof(T));
+    cudaMemPool_t pool = device_pool();
+    cudaError_t e = pool ? cudaMallocFromPoolAsync((void **)p, n * sizeof(T), pool, 0) : cudaMalloc((void **)p, n * sizeof(T));
+    if (e == cudaSuccess && pool) e = cudaStreamSynchronize(0);
     if (e != cudaSuccess) {
         *p = nullptr;
-        return fail(NULPA_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", n * sizeof(T), cudaGetErrorString(e));
+        return fail(NULPA_ENOMEM, "device allocation of %zu bytes failed: %s", n * sizeof(T), cudaGetErrorString(e));
     }
     return NULPA_OK;
 }
 
+// callers make sure no kernel still uses p (handle stream synchronised)
+void dfree(void *p) {
+    if (p) cudaFreeAsync(p, 0);
+}
+
 void free_bins(nulpa_graph *g) {
-    cudaFree(g->wrecs);
+    if (g->stream) cudaStreamSynchronize(g->stream);
+    dfree(g->wrecs);
     g->wrecs = nullptr;
-    cudaFree(g->brecs);
+    dfree(g->brecs);
     g->brecs = nullptr;
     for (int b = 0; b < 4; ++b) {
-        cudaFree(g->bin_list[b]);
+        dfree(g->bin_list[b]);
         g->bin_list[b] = nullptr;
         g->bin_n[b] = g->bin_e[b] = 0;
     }
-    cudaFree(g->chunk_g);
-    cudaFree(g->chunk_e0);
-    cudaFree(g->chunk_e1);
-    cudaFree(g->table_off);
-    cudaFree(g->gkeys);
-    cudaFree(g->gvals);
-    cudaFree(g->occ);
-    cudaFree(g->occ_n);
-    cudaFree(g->gactive);
-    cudaFree(g->gchanged);
-    cudaFree(g->gbest);
+    dfree(g->chunk_g);
+    dfree(g->chunk_e0);
+    dfree(g->chunk_e1);
+    dfree(g->table_off);
+    dfree(g->gkeys);
+    dfree(g->gvals);
+    dfree(g->occ);
+    dfree(g->occ_n);
+    dfree(g->gactive);
+    dfree(g->gchanged);
+    dfree(g->gbest);
     g->gbest = nullptr;
     g->chunk_g = nullptr;
     g->chunk_e0 = g->chunk_e1 = g->table_off = nullptr;
@@ -1607,7 +1643,7 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         std::vector<int64_t> roff(ng);
         CU(cudaMemcpyAsync(roff.data(), ddeg + ng, ng * sizeof(int64_t), cudaMemcpyDeviceToHost, g->stream));
         CU(cudaStreamSynchronize(g->stream));
-        cudaFree(ddeg);
+        dfree(ddeg);
         std::vector<int32_t> cg;
         std::vector<int64_t> c0, c1, toff(ng);
         int64_t slots = 0;
@@ -1642,9 +1678,9 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CU(cudaMemsetAsync(g->occ_n, 0, ng * sizeof(int32_t), g->stream));
     }
     CU(cudaStreamSynchronize(g->stream));
-    cudaFree(counts);
-    cudaFree(totals);
-    cudaFree(edges);
+    dfree(counts);
+    dfree(totals);
+    dfree(edges);
     for (int b = 0; b < 4; ++b) {
         g->stats.bin_vertices[b] = g->bin_n[b];
         g->stats.bin_edges[b] = g->bin_e[b];
@@ -2215,7 +2251,7 @@ int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double 
     double sigma = 0, two_m = 0;
     int r = nulpa_modularity_partial(g, lab, &sigma, &two_m, g->Sigma);
     if (r == NULPA_OK) r = nulpa_modularity_finish(g, g->Sigma, sigma, two_m, q);
-    cudaFree(tmp);
+    dfree(tmp);
     return r;
 }
 
@@ -2237,19 +2273,19 @@ int nulpa_destroy(nulpa_graph *g) {
     if (g->stream) cudaStreamSynchronize(g->stream);
     free_bins(g);
     if (g->own_csr) {
-        cudaFree(g->offsets);
-        cudaFree(g->indices);
-        cudaFree(g->weights);
+        dfree(g->offsets);
+        dfree(g->indices);
+        dfree(g->weights);
     }
-    cudaFree(g->own_labels);
-    cudaFree(g->own_flags);
-    cudaFree(g->labels_prev);
-    cudaFree(g->flags_prev);
-    cudaFree(g->ctr);
+    dfree(g->own_labels);
+    dfree(g->own_flags);
+    dfree(g->labels_prev);
+    dfree(g->flags_prev);
+    dfree(g->ctr);
     if (g->ctr_host) cudaFreeHost(g->ctr_host);
-    cudaFree(g->Sigma);
-    cudaFree(g->macc);
-    cudaFree(g->Kdeg);
+    dfree(g->Sigma);
+    dfree(g->macc);
+    dfree(g->Kdeg);
     if (g->hi) {
         cudaStreamSynchronize(g->hi);
         cudaStreamDestroy(g->hi);
