@@ -664,25 +664,16 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
     const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
     const int64_t ng = (nrec + 31) / 32;
-    // Balanced block-cyclic schedule: R full rounds in which every warp takes
-    // K consecutive groups (round r, warp gw: groups r*nw*K + gw*K + [0, K)),
-    // then a last round splitting the remaining groups evenly (K2 per warp).
-    // Within its blocks a warp walks consecutive rows in order, so labels
-    // propagate along ID order as in the sequential Algorithm 1 (modularity);
-    // K = 1 is the plain strided schedule.
+    // Record groups of this warp.  K = 1: static strided, groups gw, gw + nw, ...
+    // K > 1: dynamic (guided) chunks -- a warp grabs its next chunk of
+    // min(K, groups left / nw) consecutive groups from a global counter, so
+    // it walks runs of up to 32K consecutive rows in order (labels propagate
+    // along ID order as in the sequential Algorithm 1: modularity) and the
+    // chunks shrink toward the end of the sweep.  (A static K-block schedule
+    // gave each warp only ~2 blocks per sweep and left a long tail.)
     const int64_t K = SLOTS == kWarpSlots ? a.sched_block : 1;
-    const int64_t R = ng / (nw * K), rem = ng - R * nw * K, K2 = (rem + nw - 1) / nw;
-    const int64_t nq = R * K + std::max<int64_t>(0, std::min<int64_t>(K2, rem - gw * K2));
-    auto gidx = [&](int64_t q) -> int64_t {
-        return q < R * K ? (q / K) * nw * K + gw * K + q % K : R * nw * K + gw * K2 + (q - R * K);
-    };
-    // K > 1: dynamic (guided) chunks instead -- a warp grabs its next chunk of
-    // min(K, groups left / nw) groups from a global counter.  A static K-block
-    // schedule gives each warp only ~2 blocks per sweep (a block of 128 groups
-    // is ~1/2 of a warp's sweep), so unequal block weights left a long tail
-    // (sweep 0: 26 ms vs 20 ms strided); guided chunks shrink toward the end.
     const bool dyn = K > 1;
-    int64_t cur = 0, lim = dyn ? 0 : nq;                   // static: group counter q < nq; dynamic: chunk [cur, lim)
+    int64_t cur = dyn ? 0 : gw, lim = dyn ? 0 : ng;        // static: next group cur (step nw); dynamic: chunk [cur, lim)
     unsigned long long c_ch = 0, c_che = 0;
     auto grec_next = [&]() -> VRec {                       // lane's record of the warp's next group (or empty)
         VRec z{0, 0, 0, 0};
@@ -698,8 +689,8 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
             lim = std::min<int64_t>(ng, cur + (int64_t)__shfl_sync(0xFFFFFFFFu, size, 0));
         }
         if (cur >= lim) return z;
-        const int64_t i = (dyn ? cur : gidx(cur)) * 32 + lane;
-        ++cur;
+        const int64_t i = cur * 32 + lane;
+        cur += dyn ? 1 : nw;
         return i < nrec ? recs[i] : z;
     };
     auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };

@@ -2,12 +2,14 @@
 page (instructions executed, stall samples per instruction) with the line
 table of the cubin (nvdisasm -g), so hot spots read as nulpa.cu lines.
 
-usage: python scripts/ncu_lines.py <report.ncu-rep> <mangled-kernel-substring> [top]
+usage: python scripts/ncu_lines.py <report.ncu-rep> <mangled-kernel-substring> [top] [launch-index]
+(BY=0 sorts by stall samples, BY=1 (default) by instructions executed)
 """
 import collections, csv, io, os, re, subprocess, sys, tempfile
 
 rep, kname = sys.argv[1], sys.argv[2]
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 40
+launch = sys.argv[4] if len(sys.argv) > 4 else "0"
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 lib = os.path.join(ROOT, "paper_conf_ipps_sahunk25_b200", "libnulpa.so")
 
@@ -31,7 +33,8 @@ for ln in dis.splitlines():
     if m and cur_fn and kname in cur_fn:
         line_of[int(m.group(1), 16)] = cur_line
 
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass",
+                      "--launch-skip", launch, "--launch-count", "1"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 hi = next(i for i, r in enumerate(rows) if r and r[0] == "Address")
