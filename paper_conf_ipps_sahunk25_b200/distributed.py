@@ -9,8 +9,8 @@ against a REPLICATED label vector, then
   * the labels of every rank's range are exchanged with an all-gather
     (``all_gather_into_tensor`` over a padded [P, max_rows] staging buffer);
   * the "unprocessed" marks a rank set on other ranks' vertices are merged
-    with an all-reduce(MAX) of the flag vector, after which each rank keeps
-    only the flags of its own rows authoritative;
+    with a reduce-scatter(MAX) over the same padded layout: each rank
+    receives the maximum of everybody's marks for its own rows only;
   * dN is all-reduced (SUM) and Algorithm 1's tolerance / Pick-Less loop
      runs identically on every rank.
 
@@ -104,7 +104,10 @@ class CudaShardRunner:
 
 
 class Exchanger:
-    """Per-sweep exchange of labels (all-gather) and flags (all-reduce MAX)."""
+    """Per-sweep exchange of labels (all-gather) and flags (reduce-scatter
+    MAX: a rank needs only its own rows' flags, so each rank receives the
+    element-wise maximum of everybody's marks for its range -- half the bytes
+    of an all-reduce of the whole flag vector)."""
 
     def __init__(self, runner, group=None):
         self.r = runner
@@ -117,6 +120,8 @@ class Exchanger:
         dev = runner.labels.device
         self.stage_in = torch.empty(self.maxrows, dtype=torch.int32, device=dev)
         self.stage_out = torch.empty(self.world * self.maxrows, dtype=torch.int32, device=dev)
+        self.fstage_in = torch.zeros(self.world * self.maxrows, dtype=torch.uint8, device=dev)
+        self.fstage_out = torch.empty(self.maxrows, dtype=torch.uint8, device=dev)
         b, e = bounds[self.rank]
         self.own = (b, e)
 
@@ -129,7 +134,13 @@ class Exchanger:
                 self.r.labels[qb:qe].copy_(self.stage_out[q * self.maxrows: q * self.maxrows + (qe - qb)])
 
     def flags(self):
-        dist.all_reduce(self.r.flags, op=dist.ReduceOp.MAX, group=self.group)
+        f = self.r.flags
+        for q, (qb, qe) in enumerate(self.bounds):
+            if qe > qb:
+                self.fstage_in[q * self.maxrows: q * self.maxrows + (qe - qb)].copy_(f[qb:qe])
+        dist.reduce_scatter_tensor(self.fstage_out, self.fstage_in, op=dist.ReduceOp.MAX, group=self.group)
+        b, e = self.own
+        f[b:e].copy_(self.fstage_out[: e - b])
         self.clear_remote_flags()
 
     def clear_remote_flags(self):
