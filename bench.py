@@ -50,6 +50,8 @@ def parse_args():
     ap.add_argument("--extra", action="store_true", help="also time the unit-weight fast path and sync mode")
     ap.add_argument("--param", action="append", default=[], metavar="KEY=INT",
                     help="override an nulpa_params field (experiments), e.g. --param first_sweep_block=1")
+    ap.add_argument("--distributed", action="store_true",
+                    help="use the multi-GPU driver even at one rank (launch with torchrun; tests the NCCL path)")
     ap.add_argument("--quality-runs", type=int, default=4,
                     help="extra untimed runs whose modularity is reported next to the timed run's")
     return ap.parse_args()
@@ -224,7 +226,7 @@ def run_ours(args):
         if world == 1 and args.gpus > 1:
             raise SystemExit("--gpus N > 1 must be launched with torchrun (one rank per GPU)")
     torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 or args.distributed:
         return run_distributed(args, rank, world, local)
 
     t_gen = time.perf_counter()
@@ -404,14 +406,48 @@ def run_distributed(args, rank, world, local):
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms = float(ms.item())
     q = D.modularity_distributed(runner)
+    e2e_line = None
+    if not args.no_e2e:
+        # end to end through the distributed driver's public API: every step
+        # each rank copies its shard's CSR from pinned host memory (inside
+        # CudaShardRunner), runs lpa_distributed and reads its rows' labels
+        # back to pinned host memory; max over ranks
+        hs = D.Shard(shard.offsets.cpu().pin_memory(), shard.indices.cpu().pin_memory(),
+                     None if shard.weights is None else shard.weights.cpu().pin_memory(),
+                     shard.row_begin, shard.row_end, shard.N_global, shard.M_global, shard.bounds)
+        lab_h = torch.empty(shard.row_end - shard.row_begin, dtype=torch.int32).pin_memory()
+        h2d = hs.offsets.numel() * 8 + hs.indices.numel() * 4 + (0 if hs.weights is None else hs.weights.numel() * 4)
+        times = []
+        for it in range(max(1, min(args.steps, 3)) + 1):
+            torch.cuda.synchronize()
+            dist.barrier()
+            t0 = time.perf_counter()
+            r2 = D.CudaShardRunner(hs)
+            D.lpa_distributed(r2)
+            lab_h.copy_(r2.labels[shard.row_begin:shard.row_end])
+            torch.cuda.synchronize()
+            t1 = time.perf_counter()
+            r2.g.close()
+            del r2
+            if it > 0:
+                times.append(t1 - t0)
+        sec = torch.tensor([sum(times) / len(times)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(sec, op=dist.ReduceOp.MAX)
+        b_in = torch.tensor([h2d], dtype=torch.int64, device="cuda")
+        dist.all_reduce(b_in, op=dist.ReduceOp.SUM)
+        e2e_line = {"value": shard.M_global / float(sec.item()), "unit": "edges/s",
+                    "h2d_bytes_per_step": int(b_in.item()), "d2h_bytes_per_step": shard.N_global * 4,
+                    "ms_per_step": float(sec.item()) * 1e3, "steps": len(times)}
     if rank == 0:
         line = {"metric": METRIC, "value": shard.M_global / (ms / 1e3), "unit": "edges/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": {"workload": args.config, "N": shard.N_global, "M": shard.M_global, "weights": args.weights,
-                           "parallelism": f"vertex range split by edge count over {world} GPUs, NCCL all-gather of labels per sweep"},
+                           "parallelism": f"vertex range split by edge count over {world} GPUs; per sweep NCCL all-gather of labels, reduce-scatter(MAX) of flags"},
                 "iterations": res["iterations"], "changed": res["changed"], "modularity": q,
                 "gpu_launches": launches, "clocks": ck}
+        if e2e_line:
+            line["e2e"] = e2e_line
         print(json.dumps(line), flush=True)
     dist.barrier()
     dist.destroy_process_group()
