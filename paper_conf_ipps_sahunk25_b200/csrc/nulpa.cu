@@ -1816,7 +1816,15 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs,
                                                                           0xFFFFFFFFu, nullptr, nullptr);
             if (mid_fork) CU(cudaEventRecord(g->ev_mid, cs));
-            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * kWarpCtasPerSm, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
+            // first-sweep runs of up to K groups need >= K*32 rows per warp: on a
+            // small bin (a row shard of a multi-GPU run) launch fewer CTAs per SM
+            // so each warp still walks long runs (modularity)
+            int ctas = kWarpCtasPerSm;
+            if (a.sched_block > 1 && g->sweeps_since_reset == 0) {
+                const int64_t per = (int64_t)a.sched_block * 32 * kWarpWarps * sms;
+                ctas = (int)std::max<int64_t>(1, std::min<int64_t>(kWarpCtasPerSm, n / per));
+            }
+            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * ctas, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
                                                                                           ctr + kCtrSchedW);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
