@@ -76,9 +76,10 @@ typedef struct nulpa_params {
                                     warp-bin frontier (they fill the warp bin's tail; +1%)      */
     int32_t wide_degree;         /* within the block bin: degree < this -> one warp per vertex
                                     with a warp-private 1023-slot shared-memory table (load
-                                    <= 1/2); degree >= this -> one CTA per vertex.  Range
-                                    [1, 512]; <= block_degree sends the whole bin to the CTA
-                                    kernel.  B200 default 512                                   */
+                                    <= 1/2 at 512); degree >= this -> one CTA per vertex.
+                                    Range [1, 1024] (distinct labels <= D <= 1023 = p1, so R5's
+                                    linear continuation always finds a slot); <= block_degree
+                                    sends the whole bin to the CTA kernel.  B200 default 512    */
     int32_t first_sweep_block;   /* warp-bin schedule of the first sweep after a reset: each warp
                                     walks blocks of this many consecutive 32-vertex record groups
                                     (balanced block-cyclic; 1 = strided).  Larger blocks let labels

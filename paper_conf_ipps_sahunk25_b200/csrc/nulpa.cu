@@ -641,10 +641,22 @@ constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers p
 // The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
 // tables (8 KB per warp, p1 = 1023), 4 warps per CTA, 6 CTAs (24 warps) per SM.
 constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
+// Records per group (the unit a warp takes from the frontier): 32 in the warp
+// bin; the wide variant takes groups of NULPA_WIDE_GROUP (4) records from a
+// dynamic counter -- its ~200K vertices of degree 256..511 in 32-record groups
+// were only ~1.8 groups per warp, and the static strided split left half the
+// warps idle for the second half of the launch.
+#ifndef NULPA_WIDE_GROUP
+#define NULPA_WIDE_GROUP 4
+#endif
+#ifndef NULPA_WIDE_K
+#define NULPA_WIDE_K 2                   // wide schedule: guided chunks of <= this many groups
+#endif
 template <int SLOTS> struct WarpCfg {
     static constexpr int warps = SLOTS == kWarpSlots ? kWarpWarps : kWideWarps;
     static constexpr int ctas = SLOTS == kWarpSlots ? kWarpCtasPerSm : kWideCtasPerSm;
     static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step
+    static constexpr int group = SLOTS == kWarpSlots ? 32 : NULPA_WIDE_GROUP;
 };
 
 template <bool SYNC, bool W, int TIE, int SLOTS>
@@ -653,6 +665,8 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
            unsigned long long *sched) {
     constexpr int kWarpWarps = WarpCfg<SLOTS>::warps;
     constexpr int U = WarpCfg<SLOTS>::unroll;
+    constexpr int G = WarpCfg<SLOTS>::group;
+    static_assert(G >= 1 && G <= 32 && (G & (G - 1)) == 0, "group size: power of two <= 32");
     __shared__ __align__(16) uint64_t s_tab[kWarpWarps][SLOTS];
     __shared__ VRec s_ring[kWarpWarps][2][32];
     __shared__ unsigned long long bctr[2];
@@ -663,7 +677,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     const int64_t nrec = (int64_t)*count;
     const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
     const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
-    const int64_t ng = (nrec + 31) / 32;
+    const int64_t ng = (nrec + G - 1) / G;
     // Record groups of this warp.  K = 1: static strided, groups gw, gw + nw, ...
     // K > 1: dynamic (guided) chunks -- a warp grabs its next chunk of
     // min(K, groups left / nw) consecutive groups from a global counter, so
@@ -671,7 +685,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     // along ID order as in the sequential Algorithm 1: modularity) and the
     // chunks shrink toward the end of the sweep.  (A static K-block schedule
     // gave each warp only ~2 blocks per sweep and left a long tail.)
-    const int64_t K = SLOTS == kWarpSlots ? a.sched_block : 1;
+    const int64_t K = SLOTS == kWarpSlots ? a.sched_block : NULPA_WIDE_K;
     const bool dyn = K > 1;
     int64_t cur = dyn ? 0 : gw, lim = dyn ? 0 : ng;        // static: next group cur (step nw); dynamic: chunk [cur, lim)
     unsigned long long c_ch = 0, c_che = 0;
@@ -689,11 +703,11 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
             lim = std::min<int64_t>(ng, cur + (int64_t)__shfl_sync(0xFFFFFFFFu, size, 0));
         }
         if (cur >= lim) return z;
-        const int64_t i = cur * 32 + lane;
+        const int64_t i = cur * G + lane;
         cur += dyn ? 1 : nw;
-        return i < nrec ? recs[i] : z;
+        return lane < G && i < nrec ? recs[i] : z;
     };
-    auto rrec = [&](int m) -> VRec { return s_ring[wid][(m >> 5) & 1][m & 31]; };
+    auto rrec = [&](int m) -> VRec { return s_ring[wid][((unsigned)m / G) & 1][m & (G - 1)]; };
     auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
     s_ring[wid][0][lane] = grec_next();                  // zero records (degree 0) past the end
@@ -737,9 +751,9 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     // one pipeline step: issue vertex n+2's row loads (s2), vertex n+1's label
     // gathers (s1), fold vertex n (s0)
     auto step = [&](int n, Stage &s0, Stage &s1, Stage &s2) {
-        if ((n & 31) == 0 && n > 0) {
-            // entering group q = n/32: group q+1 goes where group q-1 was, group q+2 is requested
-            s_ring[wid][((n >> 5) + 1) & 1][lane] = pend;
+        if ((n & (G - 1)) == 0 && n > 0) {
+            // entering group q = n/G: group q+1 goes where group q-1 was, group q+2 is requested
+            s_ring[wid][((unsigned)n / G + 1) & 1][lane] = pend;
             pend = grec_next();
             __syncwarp();
         }
@@ -1692,8 +1706,8 @@ int validate_params(const nulpa_params &p) {
     if (p.bin_order < 0 || p.bin_order > 3) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2 or 3");
     if (p.first_sweep_block < 1 || p.first_sweep_block > 1024 || p.sweep_block < 1 || p.sweep_block > 1024)
         return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [1, 1024]");
-    if (p.wide_degree < 1 || p.wide_degree > 512)
-        return fail(NULPA_EINVAL, "wide_degree must be in [1, 512] (wide warp tables hold 1023 slots)");
+    if (p.wide_degree < 1 || p.wide_degree > 1024)   // distinct labels <= D <= 1023 = p1 (R5 always finds a slot)
+        return fail(NULPA_EINVAL, "wide_degree must be in [1, 1024] (wide warp tables hold 1023 slots)");
     if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
         return fail(NULPA_EINVAL, "giant_degree must be in [block_degree, 4096] (CTA tables hold 4095 slots)");
     return NULPA_OK;

@@ -20,7 +20,8 @@ pytestmark = pytest.mark.gpu
 
 # degree-bin configurations: default; every bin (and both block-bin kernels)
 # populated on small graphs; the paper's two-kernel split (thread < 32 <=
-# block); all-warp; all-wide-warp (+ CTA kernel for degree >= 512); all-CTA
+# block); all-warp; all-wide-warp (+ CTA kernel for degree >= 512); all-wide-warp
+# up to degree 1023 (table load up to 1: the R5 continuation); all-CTA
 # (wide_degree=1); all-giant
 BINS = {
     "default": dict(),
@@ -28,6 +29,7 @@ BINS = {
     "paper": dict(switch_degree=32, block_degree=32, wide_degree=1, giant_degree=4096),
     "warp": dict(switch_degree=1, block_degree=256, giant_degree=4096),
     "wide": dict(switch_degree=1, block_degree=1, giant_degree=4096),
+    "wide_full": dict(switch_degree=1, block_degree=1, wide_degree=1024, giant_degree=4096),
     "block": dict(switch_degree=1, block_degree=1, wide_degree=1, giant_degree=4096),
     "giant": dict(switch_degree=1, block_degree=1, giant_degree=1),
     "concurrent": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40, bin_order=3),
@@ -300,7 +302,7 @@ def test_invalid_params_raise():
     with pytest.raises(nl.NulpaError):
         gg.run(max_iterations=100)
     with pytest.raises(nl.NulpaError):
-        gg.run(wide_degree=513)
+        gg.run(wide_degree=1025)
     with pytest.raises(nl.NulpaError):
         gg.run(first_sweep_block=0)
     with pytest.raises(nl.NulpaError):
