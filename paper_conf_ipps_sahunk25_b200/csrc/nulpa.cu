@@ -269,10 +269,26 @@ __device__ __forceinline__ uint64_t lds_u64(uint32_t addr) {
 __device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
     asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
 }
+// k_warp tables store the tag k + 1 for label k (labels are >= 0 and < 2^31 - 1),
+// so an empty slot (tag 0, value 0.0f) is all-zero and hashtableClear is a
+// 16-byte store of the zero register (no per-vertex register set-up).
+#ifndef NULPA_ZERO_EMPTY
+#define NULPA_ZERO_EMPTY 1
+#endif
+#if NULPA_ZERO_EMPTY
+constexpr uint32_t kTagEmpty = 0u;
+__device__ __forceinline__ uint32_t kv_tag(int32_t k) { return (uint32_t)k + 1u; }
+__device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(addr), "r"(0u) : "memory");
+}
+#else
+constexpr uint32_t kTagEmpty = 0xFFFFFFFFu;
+__device__ __forceinline__ uint32_t kv_tag(int32_t k) { return (uint32_t)k; }
 __device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
     // two empty slots: key = phi (0xFFFFFFFF), value = 0.0f
     asm volatile("st.shared.v4.u32 [%0], {%1, %2, %1, %2};" ::"r"(addr), "r"(0xFFFFFFFFu), "r"(0u) : "memory");
 }
+#endif
 __device__ __forceinline__ uint32_t cas_u32(uint32_t addr, uint32_t cmp, uint32_t val) {
     uint32_t old;
     asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(addr), "r"(cmp), "r"(val) : "memory");
@@ -449,12 +465,22 @@ constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 
 // Algorithm 2's probe sequence past the home slot (hybrid quadratic-double
 // probing, R5 linear continuation) on a one-word-per-slot table of capacity P.
+// Continues after probe t0 at slot i (t0 = 0: the home slot; t0 = 1: home + 1,
+// where the step delta_1 = 1 has become delta_2 = 2 + (k mod p2) mod P).
+#ifndef NULPA_PROBE2
+#define NULPA_PROBE2 1
+#endif
 template <uint32_t P>
-__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x) {
+__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint32_t i, int t0) {
     constexpr uint32_t p2 = 2 * P + 1;                    // R3
-    uint32_t i = (uint32_t)k % P, di = 1;
     const uint32_t km = ((uint32_t)k % p2) % P;
-    for (int t = 1;; ++t) {
+    uint32_t di = 1;
+    if (t0 == 1) {
+        di = 2 + km;
+        if (di >= P) di -= P;
+    }
+    const uint32_t tg = kv_tag(k);
+    for (int t = t0 + 1;; ++t) {
         if (t <= kMaxRetries) {
             i += di;
             if (i >= P) i -= P;
@@ -465,13 +491,13 @@ __device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x) {
             i = i + 1 == P ? 0 : i + 1;                    // R5
         }
         const uint64_t cur = lds_u64(tab + 8 * i);
-        const int32_t ck = (int32_t)(uint32_t)cur;
-        if (ck == k) {
+        const uint32_t ck = (uint32_t)cur;
+        if (ck == tg) {
             const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
             sts_f32(tab + 8 * i + 4, V);
             return V;
         }
-        if (ck == kEmpty && cas_u32(tab + 8 * i, 0xFFFFFFFFu, (uint32_t)k) == 0xFFFFFFFFu) {
+        if (ck == kTagEmpty && cas_u32(tab + 8 * i, kTagEmpty, tg) == kTagEmpty) {
             sts_f32(tab + 8 * i + 4, x);
             return x;
         }
@@ -484,18 +510,38 @@ __device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x) {
 template <uint32_t P>
 __device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, float x) {
     const uint32_t i = (uint32_t)k % P;
+    const uint32_t tg = kv_tag(k);
     const uint64_t cur = lds_u64(tab + 8 * i);
-    const int32_t ck = (int32_t)(uint32_t)cur;
-    if (ck == k) {
+    const uint32_t ck = (uint32_t)cur;
+    if (ck == tg) {
         const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
         sts_f32(tab + 8 * i + 4, V);
         return V;
     }
-    if (ck == kEmpty && cas_u32(tab + 8 * i, 0xFFFFFFFFu, (uint32_t)k) == 0xFFFFFFFFu) {
+    if (ck == kTagEmpty && cas_u32(tab + 8 * i, kTagEmpty, tg) == kTagEmpty) {
         sts_f32(tab + 8 * i + 4, x);
         return x;
     }
-    return kv_add_slow<P>(tab, k, x);
+#if NULPA_PROBE2
+    // Probe 1 of the sequence (delta_0 = 1: the next slot) inline: with ~25
+    // leaders per batch some lane almost always collides at home in the first
+    // sweep, and the warp would take the out-of-line path together.
+    const uint32_t i1 = i + 1 == P ? 0u : i + 1;
+    const uint64_t cur1 = lds_u64(tab + 8 * i1);
+    const uint32_t ck1 = (uint32_t)cur1;
+    if (ck1 == tg) {
+        const float V = __fadd_rn(__uint_as_float((uint32_t)(cur1 >> 32)), x);
+        sts_f32(tab + 8 * i1 + 4, V);
+        return V;
+    }
+    if (ck1 == kTagEmpty && cas_u32(tab + 8 * i1, kTagEmpty, tg) == kTagEmpty) {
+        sts_f32(tab + 8 * i1 + 4, x);
+        return x;
+    }
+    return kv_add_slow<P>(tab, k, x, i1, 1);
+#else
+    return kv_add_slow<P>(tab, k, x, i, 0);
+#endif
 }
 
 // ---------------------------------------------------------------------------
@@ -668,7 +714,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     constexpr int G = WarpCfg<SLOTS>::group;
     static_assert(G >= 1 && G <= 32 && (G & (G - 1)) == 0, "group size: power of two <= 32");
     __shared__ __align__(16) uint64_t s_tab[kWarpWarps][SLOTS];
-    __shared__ VRec s_ring[kWarpWarps][2][32];
+    __shared__ VRec s_ring[kWarpWarps][2 * G];        // two groups; record m sits at m mod 2G
     __shared__ unsigned long long bctr[2];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const uint32_t tab = (uint32_t)__cvta_generic_to_shared(&s_tab[wid][0]);
@@ -707,11 +753,16 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         cur += dyn ? 1 : nw;
         return lane < G && i < nrec ? recs[i] : z;
     };
-    auto rrec = [&](int m) -> VRec { return s_ring[wid][((unsigned)m / G) & 1][m & (G - 1)]; };
+    auto rrec = [&](int m) -> VRec { return s_ring[wid][m & (2 * G - 1)]; };
     auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
-    s_ring[wid][0][lane] = grec_next();                  // zero records (degree 0) past the end
-    s_ring[wid][1][lane] = grec_next();
+    {
+        const VRec r0 = grec_next(), r1 = grec_next();   // zero records (degree 0) past the end
+        if (lane < G) {
+            s_ring[wid][lane] = r0;
+            s_ring[wid][G + lane] = r1;
+        }
+    }
     VRec pend = grec_next();
     __syncwarp();
     // pipeline registers of one vertex: entries lane and lane+32 of its row
@@ -753,7 +804,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     auto step = [&](int n, Stage &s0, Stage &s1, Stage &s2) {
         if ((n & (G - 1)) == 0 && n > 0) {
             // entering group q = n/G: group q+1 goes where group q-1 was, group q+2 is requested
-            s_ring[wid][((unsigned)n / G + 1) & 1][lane] = pend;
+            if (lane < G) s_ring[wid][(n + G + lane) & (2 * G - 1)] = pend;
             pend = grec_next();
             __syncwarp();
         }
