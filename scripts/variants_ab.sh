@@ -4,7 +4,7 @@
 SEEDS=${2:-"0 1"}
 for spec in $1; do
   name=${spec%%:*}; defs=${spec#*:}
-  python paper_conf_ipps_sahunk25_b200/build.py --out /tmp/nulpa_$name.so $defs > /dev/null || { echo "build $name failed"; continue; }
+  python paper_conf_ipps_sahunk25_b200/build.py --out /tmp/nulpa_$name.so ${defs//,/ } > /dev/null || { echo "build $name failed"; continue; }
   echo "== $name ($defs)"
   NULPA_LIB=/tmp/nulpa_$name.so python scripts/kbench.py --async-too 2>&1 | tail -n 4
   for s in $SEEDS; do
