@@ -143,10 +143,11 @@ def test_web_2200m_quality_vs_full_oracle():
     are recorded; the test asserts the neighbour-label invariant and records
     the comparison (NULPA_FULLSIZE_OUT: JSON path)."""
     import json, time
-    g = synth.make("web_40m_2200m", device="cuda")
+    seed = int(os.environ.get("NULPA_FULLSIZE_SEED", "0"))
+    g = synth.make("web_40m_2200m", device="cuda", seed=seed)
     gg = nl.Graph(g.offsets, g.indices, None)
     runs = []
-    for r in range(6):
+    for r in range(int(os.environ.get("NULPA_FULLSIZE_RUNS", "6"))):
         st = gg.run()
         runs.append(dict(modularity=gg.modularity(), iterations=st["iterations"], changed=st["changed"]))
     sync_st = gg.run(mode=nl.SYNC)
@@ -158,7 +159,7 @@ def test_web_2200m_quality_vs_full_oracle():
     q_or = oracle.modularity(h, C)
     q_or_gpu = gg.modularity(torch.from_numpy(C).cuda())
     assert abs(q_or - q_or_gpu) < 1e-6          # Eq. 1 on the GPU agrees with the oracle's
-    out = dict(graph="web_40m_2200m seed 0, unit weights", N=g.N, M=g.M,
+    out = dict(graph=f"web_40m_2200m seed {seed}, unit weights", N=g.N, M=g.M,
                gpu_async_runs=runs, gpu_sync=dict(modularity=sync_q, iterations=sync_st["iterations"]),
                oracle=dict(modularity=q_or, iterations=it, changed=[int(x) for x in dN], seconds=round(t_or, 1)))
     print(json.dumps(out))
