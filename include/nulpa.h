@@ -87,10 +87,11 @@ typedef struct nulpa_params {
                                     Algorithm 1 (better modularity) at some memory-latency cost.
                                     Range [1, 1024]; default 128    */
     int32_t sweep_block;         /* the same for every later sweep; default 4.  Any value > 1
-                                    hands out guided chunks of min(block, max(32, groups left /
-                                    warps)) from a global counter (balance; the floor of 32
-                                    groups keeps first-sweep runs >= 1024 rows, see DESIGN.md
-                                    "Quality notes"); 1 is the static strided schedule          */
+                                    hands out guided chunks of min(block, max(block / 4, groups
+                                    left / warps)) from a global counter (balance; the floor
+                                    keeps first-sweep runs >= 1024 rows at the default 128, see
+                                    DESIGN.md "Quality notes"); 1 is the static strided
+                                    schedule                                                    */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0

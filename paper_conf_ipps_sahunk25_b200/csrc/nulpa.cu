@@ -680,12 +680,12 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #define NULPA_GUIDED_C 1                 // guided chunk = min(K, groups left / (C * warps)) ...
 #endif
 #ifndef NULPA_GUIDED_DIV
-#define NULPA_GUIDED_DIV 0               // experiment: floor = K / this instead of min(K, NULPA_GUIDED_MIN)
+#define NULPA_GUIDED_DIV 4               // ... but at least K / this (0: min(K, NULPA_GUIDED_MIN)): the
+                                         // first sweep's chunks (K = 128) never drop below 32 groups
+                                         // (DESIGN.md "Quality notes"); later sweeps (K = 4) keep 1
 #endif
 #ifndef NULPA_GUIDED_MIN
-#define NULPA_GUIDED_MIN 32              // ... but at least min(K, this): with 1, the shrinking
-                                         // first-sweep chunks at the end of the sweep let labels
-                                         // flood (Q 0.815 in 1 of 9 runs, seed 0)
+#define NULPA_GUIDED_MIN 1
 #endif
 
 constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
