@@ -85,11 +85,11 @@ typedef struct nulpa_params {
                                     (balanced block-cyclic; 1 = strided).  Larger blocks let labels
                                     propagate along ID order within a warp as in the sequential
                                     Algorithm 1 (better modularity) at some memory-latency cost.
-                                    Range [1, 1024]; default 128    */
+                                    Range [1, 1024]; default 192    */
     int32_t sweep_block;         /* the same for every later sweep; default 4.  Any value > 1
                                     hands out guided chunks of min(block, max(block / 4, groups
                                     left / warps)) from a global counter (balance; the floor
-                                    keeps first-sweep runs >= 1024 rows at the default 128, see
+                                    keeps first-sweep runs >= 1536 rows at the default 192, see
                                     DESIGN.md "Quality notes"); 1 is the static strided
                                     schedule                                                    */
 } nulpa_params;

@@ -2056,7 +2056,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->tie_rule = NULPA_TIE_SMALLEST;
     p->bin_order = 1;
     p->wide_degree = 512;
-    p->first_sweep_block = 128;
+    p->first_sweep_block = 192;
     p->sweep_block = 4;
 }
 
