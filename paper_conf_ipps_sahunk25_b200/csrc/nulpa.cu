@@ -350,6 +350,7 @@ struct SweepArgs {
     int64_t row_begin;
     int pickless;
     int sched_block;           // warp-bin schedule: record groups per block (k_warp)
+    int split;                 // 1: warp-bin k_warp takes one contiguous 1/nw of the groups per warp
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 
@@ -679,6 +680,9 @@ constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_GUIDED_C
 #define NULPA_GUIDED_C 1                 // guided chunk = min(K, groups left / (C * warps)) ...
 #endif
+#ifndef NULPA_FIRST_SPLIT
+#define NULPA_FIRST_SPLIT 0              // first sweep: contiguous equal split of the warp-bin groups
+#endif
 #ifndef NULPA_GUIDED_DIV
 #define NULPA_GUIDED_DIV 4               // ... but at least K / this (0: min(K, NULPA_GUIDED_MIN)): the
                                          // first sweep's chunks (K = 128) never drop below 32 groups
@@ -737,8 +741,17 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     // chunks shrink toward the end of the sweep.  (A static K-block schedule
     // gave each warp only ~2 blocks per sweep and left a long tail.)
     const int64_t K = SLOTS == kWarpSlots ? a.sched_block : NULPA_WIDE_K;
-    const bool dyn = K > 1;
+    // split (first sweep, NULPA_FIRST_SPLIT): warp gw walks the contiguous
+    // groups [gw * ng / nw, (gw + 1) * ng / nw) -- one run per warp, the fewest
+    // run starts, no tail from chunk granularity
+    const bool split = SLOTS == kWarpSlots && a.split;
+    const bool dyn = K > 1 && !split;
     int64_t cur = dyn ? 0 : gw, lim = dyn ? 0 : ng;        // static: next group cur (step nw); dynamic: chunk [cur, lim)
+    if (split) {
+        cur = gw * ng / nw;
+        lim = (gw + 1) * ng / nw;
+    }
+    const int64_t stride = dyn || split ? 1 : nw;
     unsigned long long c_ch = 0, c_che = 0;
     auto grec_next = [&]() -> VRec {                       // lane's record of the warp's next group (or empty)
         VRec z{0, 0, 0, 0};
@@ -759,7 +772,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         }
         if (cur >= lim) return z;
         const int64_t i = cur * G + lane;
-        cur += dyn ? 1 : nw;
+        cur += stride;
         return lane < G && i < nrec ? recs[i] : z;
     };
     auto rrec = [&](int m) -> VRec { return s_ring[wid][m & (2 * G - 1)]; };
@@ -1804,6 +1817,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     a.row_begin = g->row_begin;
     a.pickless = pickless;
     a.sched_block = g->sweeps_since_reset == 0 ? p.first_sweep_block : p.sweep_block;
+    a.split = NULPA_FIRST_SPLIT && g->sweeps_since_reset == 0 && p.first_sweep_block > 1;
     a.ctr = ctr;
     if (SYNC) {
         CU(cudaMemcpyAsync(g->labels_prev, g->labels, g->n_global * sizeof(int32_t), cudaMemcpyDeviceToDevice, g->stream));
