@@ -68,12 +68,13 @@ typedef struct nulpa_params {
                                     NULPA_TIE_SLOT (1): first in the table's slot order -- smallest
                                     home slot k mod p1, then smallest label (PAPER.md:173
                                     "selects the first label with the highest associated weight") */
-    int32_t bin_order;           /* 1 (default): thread, warp, block, giant bins in that order
-                                    within a sweep (hubs last); 0: giant, block, warp, thread;
-                                    2: block + giant on a second stream, concurrent with
-                                    thread + warp; 3: warp bin on a high-priority stream, block
-                                    + giant on a low-priority stream released after the
-                                    warp-bin frontier (they fill the warp bin's tail; +1%)      */
+    int32_t bin_order;           /* 3 (default): thread bin, then the warp bin on a
+                                    high-priority stream and block + giant on a low-priority
+                                    stream released after the warp-bin frontier (they fill the
+                                    warp bin's tail: +5% at first_sweep_block 192); 1: thread,
+                                    warp, block, giant bins in that order within a sweep (hubs
+                                    last); 0: giant, block, warp, thread; 2: block + giant on a
+                                    second stream, concurrent with thread + warp              */
     int32_t wide_degree;         /* within the block bin: degree < this -> one warp per vertex
                                     with a warp-private 1023-slot shared-memory table (load
                                     <= 1/2 at 512); degree >= this -> one CTA per vertex.

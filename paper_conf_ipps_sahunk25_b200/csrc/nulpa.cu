@@ -13,8 +13,10 @@
 //   giant tables: int32 keys / float32 values / int32 occupied-slot lists,
 //   one region of p1 = nextPow2(D)-1 slots per giant vertex.
 //
-// Kernels of one sweep (lpaMove), launched on the handle's stream, by default
-// in the order thread -> warp -> block -> giant (bin_order 1, hubs last):
+// Kernels of one sweep (lpaMove): thread bin, then the warp bin on a
+// high-priority stream with block + giant on a low-priority stream filling its
+// tail (bin_order 3, default; bin_order 1 = thread -> warp -> block -> giant
+// in order on the handle's stream, hubs last):
 //   k_giant_snapshot / k_giant_accumulate / k_giant_decide / k_giant_finish
 //   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
 //   k_frontier + k_warp   compacted frontier; one warp per vertex, pipelined,
@@ -2068,7 +2070,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->reset = 1;
     p->timing = 0;
     p->tie_rule = NULPA_TIE_SMALLEST;
-    p->bin_order = 1;
+    p->bin_order = 3;
     p->wide_degree = 512;
     p->first_sweep_block = 192;
     p->sweep_block = 4;

@@ -33,6 +33,7 @@ BINS = {
     "block": dict(switch_degree=1, block_degree=1, wide_degree=1, giant_degree=4096),
     "giant": dict(switch_degree=1, block_degree=1, giant_degree=1),
     "concurrent": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40, bin_order=3),
+    "inorder": dict(switch_degree=4, block_degree=12, wide_degree=24, giant_degree=40, bin_order=1),
 }
 
 
