@@ -63,11 +63,11 @@ typedef struct nulpa_params {
     int32_t reset;               /* 1: C <- [0..N) and all vertices unprocessed first;
                                     0: continue from the current labels / flags               */
     int32_t timing;              /* 1: time every kernel with CUDA events (nulpa_get_stats)   */
-    int32_t tie_rule;            /* order among labels of equal weight (R6):
-                                    NULPA_TIE_SMALLEST (0): smallest label (north star);
-                                    NULPA_TIE_SLOT (1): first in the table's slot order -- smallest
-                                    home slot k mod p1, then smallest label (PAPER.md:173
-                                    "selects the first label with the highest associated weight") */
+    int32_t tie_rule;            /* order among labels of equal weight (R6): must be
+                                    NULPA_TIE_SMALLEST (0) -- the smallest label wins (north
+                                    star "ties broken by smallest label"; "the
+                                    first label with the highest associated weight").  Any other
+                                    value is rejected with NULPA_EINVAL                          */
     int32_t bin_order;           /* 3 (default): thread bin, then the warp bin on a
                                     high-priority stream and block + giant on a low-priority
                                     stream released after the warp-bin frontier (they fill the
@@ -96,7 +96,6 @@ typedef struct nulpa_params {
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0
-#define NULPA_TIE_SLOT 1
 
 /* Statistics of the last nulpa_run (or accumulated nulpa_sweep calls since
  * the last reset).  Bins: 0 thread, 1 warp, 2 block, 3 giant. */
@@ -133,6 +132,9 @@ void nulpa_default_params(nulpa_params *p);
  *              by the handle (copy enqueued on `stream`; the host arrays may
  *              be reused once nulpa_create returns).
  *   stream   : cudaStream_t for all work of this handle.
+ * Errors: NULPA_EINVAL for null/inconsistent sizes, offsets[0] != 0, or any
+ * weight that is negative, NaN or infinite (R12: one device pass checks
+ * them); NULPA_ENOMEM / NULPA_ECUDA from allocation / copies.
  * Builds the degree-binned frontier (row a1) with the default switch degrees;
  * nulpa_run rebuilds it if other switch degrees are requested.
  * Labels start as C = [0..n_global), all vertices unprocessed. */
@@ -164,7 +166,8 @@ int nulpa_reset(nulpa_graph *g);
 int nulpa_labels(nulpa_graph *g, int32_t *out, int memkind);
 
 /* Overwrite the labels (n_global int32 from `in` in `memkind` memory) and
- * the unprocessed flags (n_global uint8, or NULL = all unprocessed). */
+ * the unprocessed flags (n_global uint8, or NULL = all unprocessed).
+ * NULPA_EINVAL (state unchanged) if any label is outside [0, n_global). */
 int nulpa_set_labels(nulpa_graph *g, const int32_t *in, const uint8_t *flags, int memkind);
 
 /* Copy the unprocessed flags (n_global uint8) to `out`. */
@@ -172,7 +175,8 @@ int nulpa_flags(nulpa_graph *g, uint8_t *out, int memkind);
 
 /* Modularity Q of `labels` (n_global int32 in [0, n_global), memkind; NULL =
  * the handle's current labels), Eq. 1 second form (R11), float64
- * accumulation.  Requires a whole graph (n_rows == n_global). */
+ * accumulation.  Requires a whole graph (n_rows == n_global).  NULPA_EINVAL
+ * if any label is outside [0, n_global) (labels index the community sums). */
 int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double *q);
 
 /* Shard pieces of the modularity for the multi-GPU driver: adds this
@@ -185,6 +189,14 @@ int nulpa_modularity_finish(nulpa_graph *g, const double *Sigma_device, double s
                             double two_m, double *q);
 
 int nulpa_get_stats(nulpa_graph *g, nulpa_stats *out);
+
+/* Return the device memory that destroyed handles left in the library's
+ * stream-ordered pool on the current device to the driver.  Handles keep
+ * their memory in a per-device pool that retains up to 48 GB after
+ * nulpa_destroy (so create/destroy cycles of the same size reuse it instead
+ * of paying cudaMalloc/cudaFree of the CSR copy); call this before handing
+ * the memory to another allocator.  Live handles are unaffected. */
+int nulpa_release_memory(void);
 
 /* Device pointers of the current label / flag vectors (for zero-copy
  * wrapping by the binding).  Valid until the next nulpa_* call. */

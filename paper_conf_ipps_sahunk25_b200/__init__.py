@@ -20,7 +20,7 @@ __all__ = [
     "NulpaError", "Params", "Stats", "Graph", "lpa", "load_library", "library_path",
     "nulpa_create", "nulpa_run", "nulpa_sweep", "nulpa_labels", "nulpa_set_labels", "nulpa_flags",
     "nulpa_modularity", "nulpa_modularity_partial", "nulpa_modularity_finish", "nulpa_reset",
-    "nulpa_bind_state", "nulpa_get_stats", "nulpa_destroy", "nulpa_default_params", "nulpa_version",
+    "nulpa_bind_state", "nulpa_get_stats", "nulpa_release_memory", "nulpa_destroy", "nulpa_default_params", "nulpa_version",
     "ASYNC", "SYNC", "MEM_HOST", "MEM_DEVICE",
 ]
 
@@ -29,7 +29,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.environ.get("NULPA_LIB") or os.path.join(_PKG, "libnulpa.so")
 
 ASYNC, SYNC = 0, 1
-TIE_SMALLEST, TIE_SLOT = 0, 1
+TIE_SMALLEST = 0            # the only tie rule: smallest label (R6)
 MEM_HOST, MEM_DEVICE = 0, 1
 BINS = ("thread", "warp", "block", "giant")
 
@@ -122,6 +122,7 @@ def load_library():
         "nulpa_get_stats": (ctypes.c_int, [vp, P(Stats)]),
         "nulpa_state_pointers": (ctypes.c_int, [vp, P(vp), P(vp)]),
         "nulpa_destroy": (ctypes.c_int, [vp]),
+        "nulpa_release_memory": (ctypes.c_int, []),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -240,6 +241,11 @@ def nulpa_bind_state(h, labels_device, flags_device):
     _check(load_library().nulpa_bind_state(h, _ptr(labels_device), _ptr(flags_device)))
 
 
+def nulpa_release_memory():
+    """Return pooled device memory of destroyed handles to the driver."""
+    _check(load_library().nulpa_release_memory())
+
+
 def nulpa_get_stats(h) -> Stats:
     st = Stats()
     _check(load_library().nulpa_get_stats(h, ctypes.byref(st)))
@@ -273,6 +279,7 @@ class Graph:
         if getattr(self, "h", None):
             nulpa_destroy(self.h)
             self.h = None
+            nulpa_release_memory()          # hand the pooled memory back (torch may need it next)
 
     def __del__(self):
         try:

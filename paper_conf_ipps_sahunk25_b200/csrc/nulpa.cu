@@ -127,39 +127,13 @@ struct Hash {
     }
 };
 
-// Tie order among labels of equal weight (R6).  Rule 0 (north star):
-// smallest label.  Rule 1 ("the first label with the highest
-// associated weight", read as first in the table's slot order): smallest home
-// slot k mod p1, then smallest label.  Both are independent of insertion
-// order.  rank(k) maps k to a 32-bit integer whose order is the tie order:
-// rule 1 uses (k mod p1) * Q + (k div p1) with Q = floor((2^31-1)/p1) + 1,
-// a bijection onto [0, p1*Q) < 2^32; (k div p1) is the exact division
-// (k - k mod p1) * p1^-1 mod 2^32 (p1 = 2^a - 1 is odd).
-template <int RULE>
+// Tie order among labels of equal weight (R6, north star): the smallest
+// label.  rank(k) maps k to an integer whose order is the tie order
+// (identity); kept as a type so the argmax code reads as the rule it applies.
 struct TieOrder {
-    uint32_t p1, Q, inv;
-    uint64_t m1;
-    __device__ __forceinline__ void init(const Hash &h) {
-        if (RULE) {
-            p1 = h.p1;
-            m1 = h.m1;
-            Q = p1 ? 0x7FFFFFFFu / p1 + 1 : 1;
-            uint32_t x = p1;                       // Newton: x <- x (2 - p1 x)
-#pragma unroll
-            for (int i = 0; i < 5; ++i) x *= 2u - p1 * x;
-            inv = x;
-        }
-    }
-    __device__ __forceinline__ uint32_t rank(int32_t k) const {
-        if (!RULE) return (uint32_t)k;
-        const uint32_t home = fastmod((uint32_t)k, m1, p1);
-        return home * Q + ((uint32_t)k - home) * inv;
-    }
-    __device__ __forceinline__ int32_t unrank(uint32_t t) const {
-        if (!RULE) return (int32_t)t;
-        const uint32_t home = t / Q;
-        return (int32_t)((t - home * Q) * p1 + home);
-    }
+    __device__ __forceinline__ void init(const struct Hash &) {}
+    __device__ __forceinline__ uint32_t rank(int32_t k) const { return (uint32_t)k; }
+    __device__ __forceinline__ int32_t unrank(uint32_t t) const { return (int32_t)t; }
 };
 
 // hashtableAccumulate, Algorithm 2, the SHARED branch:
@@ -300,12 +274,10 @@ __device__ __forceinline__ uint32_t cas_u32(uint32_t addr, uint32_t cmp, uint32_
 // (weight, tie rank) packed so that an unsigned max gives the largest weight
 // and, among equal weights, the label first in tie order (R6; R12: weights
 // >= 0 so IEEE bit patterns order like the values).  0 = no candidate.
-template <int RULE>
-__device__ __forceinline__ uint64_t pack_cand(float w, int32_t k, const TieOrder<RULE> &to) {
+__device__ __forceinline__ uint64_t pack_cand(float w, int32_t k, const TieOrder &to) {
     return ((uint64_t)__float_as_uint(w) << 32) | (uint64_t)(0xFFFFFFFFu - to.rank(k));
 }
-template <int RULE>
-__device__ __forceinline__ int32_t cand_label(uint64_t c, const TieOrder<RULE> &to) {
+__device__ __forceinline__ int32_t cand_label(uint64_t c, const TieOrder &to) {
     return to.unrank(0xFFFFFFFFu - (uint32_t)(c & 0xFFFFFFFFu));
 }
 __device__ __forceinline__ uint64_t warp_max_u64(uint64_t x) {
@@ -391,7 +363,7 @@ __device__ __forceinline__ void block_count(unsigned long long *ctr, unsigned lo
 // lab[m] == lab[k], taken in CSR order (bit-identical to a sequential
 // float32 hashtable accumulation).
 // ---------------------------------------------------------------------------
-template <bool SYNC, bool W, int TIE, int MAXD>
+template <bool SYNC, bool W, int MAXD>
 __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const int32_t *__restrict__ list,
                                                            int64_t n) {
     __shared__ unsigned long long bctr[4];
@@ -424,7 +396,7 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
             }
             Hash h;
             h.init(deg);
-            TieOrder<TIE> to;
+            TieOrder to;
             to.init(h);
             uint64_t best = 0;
 #pragma unroll
@@ -716,7 +688,7 @@ template <int SLOTS> struct WarpCfg {
     static constexpr int group = SLOTS == kWarpSlots ? 32 : NULPA_WIDE_GROUP;
 };
 
-template <bool SYNC, bool W, int TIE, int SLOTS>
+template <bool SYNC, bool W, int SLOTS>
 __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ctas)
     k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin,
            unsigned long long *sched) {
@@ -841,7 +813,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         const int64_t vk = rc.r + a.row_begin;
         Hash h;
         h.init(dk);
-        TieOrder<TIE> to;
+        TieOrder to;
         to.init(h);
         uint32_t bw = 0;
         int32_t bk = 0;
@@ -955,7 +927,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
 // ---------------------------------------------------------------------------
 constexpr int kBlkThreads = 128;
 
-template <bool SYNC, bool W, int TIE>
+template <bool SYNC, bool W>
 __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *__restrict__ recs,
                                                         const unsigned long long *__restrict__ count) {
     extern __shared__ int32_t dyn[];
@@ -999,7 +971,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
                 Hv[q] = 0.0f;
             }
             __syncthreads();
-            TieOrder<TIE> to;
+            TieOrder to;
             to.init(h);
             uint32_t bw = 0;
             int32_t bk = 0;
@@ -1121,7 +1093,7 @@ __global__ void k_giant_snapshot(SweepArgs a, GiantArgs g, int64_t ng) {
     if (!SYNC && f) a.flag_in[v] = 0;
 }
 
-template <bool SYNC, bool W, int TIE>
+template <bool SYNC, bool W>
 __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a, GiantArgs g) {
     extern __shared__ int32_t dyn[];
     int32_t *Hk = dyn;
@@ -1187,7 +1159,7 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
     __syncthreads();
     Hash hg;
     hg.init((uint32_t)(a.offsets[r + 1] - a.offsets[r]));
-    TieOrder<TIE> to;
+    TieOrder to;
     to.init(hg);
     int32_t *gk = g.keys + g.table_off[gi];
     float *gv = g.vals + g.table_off[gi];
@@ -1215,7 +1187,7 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
 }
 
 // the move rule for every giant vertex (one thread each)
-template <bool SYNC, int TIE>
+template <bool SYNC>
 __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     const int64_t gi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (gi >= ng || !g.active[gi]) return;
@@ -1224,7 +1196,7 @@ __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     const int64_t deg = a.offsets[r + 1] - a.offsets[r];
     Hash h;
     h.init((uint32_t)deg);
-    TieOrder<TIE> to;
+    TieOrder to;
     to.init(h);
     const unsigned long long b = g.best[gi];
     const int32_t cs = b ? cand_label(b, to) : kEmpty;
@@ -1512,15 +1484,38 @@ __global__ void __launch_bounds__(256) k_mod_finish(double *Sigma, int64_t n, do
     }
 }
 
+// SM count of the current device (cached per device ordinal)
 int num_sms() {
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
+    static int sms[64] = {};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (!sms[dev]) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        sms[dev] = n > 0 ? n : 148;
     }
-    return sms;
+    return sms[dev];
+}
+
+// Input validation kernels (R12 and the label range of the C ABI).
+// bad[0] += number of weights that are negative, NaN or infinite.
+__global__ void k_check_weights(const float *__restrict__ w, int64_t m, unsigned long long *bad) {
+    unsigned long long c = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+        const float x = w[i];
+        c += !(x >= 0.0f && x <= 3.402823466e38f);      // false for NaN, < 0, +inf
+    }
+    c = __reduce_add_sync(0xFFFFFFFFu, (unsigned)c);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(bad, c);
+}
+// bad[0] += number of labels outside [0, n)
+__global__ void k_check_labels(const int32_t *__restrict__ lab, int64_t n, unsigned long long *bad) {
+    unsigned c = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        c += (lab[i] < 0 || (int64_t)lab[i] >= n);
+    c = __reduce_add_sync(0xFFFFFFFFu, c);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(bad, (unsigned long long)c);
 }
 
 }  // namespace
@@ -1748,14 +1743,17 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CHECK(dalloc(&g->gactive, (size_t)ng));
         CHECK(dalloc(&g->gchanged, (size_t)ng));
         CHECK(dalloc(&g->gbest, (size_t)ng));
-        CU(cudaMemcpy(g->chunk_g, cg.data(), cg.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
-        CU(cudaMemcpy(g->chunk_e0, c0.data(), c0.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
-        CU(cudaMemcpy(g->chunk_e1, c1.data(), c1.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
-        CU(cudaMemcpy(g->table_off, toff.data(), toff.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
+        // on the handle's stream (every bin kernel is ordered after the
+        // cudaStreamSynchronize(g->stream) below; the host vectors outlive it)
+        CU(cudaMemcpyAsync(g->chunk_g, cg.data(), cg.size() * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
+        CU(cudaMemcpyAsync(g->chunk_e0, c0.data(), c0.size() * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+        CU(cudaMemcpyAsync(g->chunk_e1, c1.data(), c1.size() * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
+        CU(cudaMemcpyAsync(g->table_off, toff.data(), toff.size() * sizeof(int64_t), cudaMemcpyHostToDevice, g->stream));
         k_fill_i32<<<grid_for(slots, 256, 4096), 256, 0, g->stream>>>(g->gkeys, slots, kEmpty);
         CU(cudaGetLastError());
         CU(cudaMemsetAsync(g->gvals, 0, slots * sizeof(float), g->stream));
         CU(cudaMemsetAsync(g->occ_n, 0, ng * sizeof(int32_t), g->stream));
+        CU(cudaStreamSynchronize(g->stream));          // before cg / c0 / c1 / toff go out of scope
     }
     CU(cudaStreamSynchronize(g->stream));
     dfree(counts);
@@ -1777,7 +1775,7 @@ int validate_params(const nulpa_params &p) {
         return fail(NULPA_EINVAL, "switch_degree must be in [1, 33] (thread-per-vertex tables live in registers)");
     if (p.block_degree < p.switch_degree || p.block_degree > 256)
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
-    if (p.tie_rule != NULPA_TIE_SMALLEST && p.tie_rule != NULPA_TIE_SLOT) return fail(NULPA_EINVAL, "unknown tie_rule");
+    if (p.tie_rule != NULPA_TIE_SMALLEST) return fail(NULPA_EINVAL, "tie_rule must be NULPA_TIE_SMALLEST (0): ties go to the smallest label (R6)");
     if (p.bin_order < 0 || p.bin_order > 3) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2 or 3");
     if (p.first_sweep_block < 1 || p.first_sweep_block > 1024 || p.sweep_block < 1 || p.sweep_block > 1024)
         return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [1, 1024]");
@@ -1793,24 +1791,24 @@ int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
     return build_bins(g, p.switch_degree, p.block_degree, p.giant_degree);
 }
 
-template <bool SYNC, bool W, int TIE>
+template <bool SYNC, bool W>
 int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const int64_t n = g->bin_n[0];
     const int grid = grid_for(n, kThreadThreads);
     const int64_t md = g->bin_maxdeg[0];     // register table sized by the bin's largest degree
     if (md <= 4)
-        k_thread<SYNC, W, TIE, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else if (md <= 8)
-        k_thread<SYNC, W, TIE, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else if (md <= 16)
-        k_thread<SYNC, W, TIE, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     else
-        k_thread<SYNC, W, TIE, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
+        k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
     CU(cudaGetLastError());
     return NULPA_OK;
 }
 
-template <bool SYNC, bool W, int TIE>
+template <bool SYNC, bool W>
 int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
     SweepArgs a;
     a.offsets = g->offsets;
@@ -1858,14 +1856,11 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             ga.changed = g->gchanged;
             ga.best = g->gbest;
             const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float)) + kGiantChunk * sizeof(uint16_t);
-            static bool attr_set = false;   // one per template instantiation
-            if (!attr_set) {
-                CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W, TIE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-                attr_set = true;
-            }
+            // set on every launch: the attribute is per device, the handle may live on any
+            CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, cs>>>(a, ga, ng);
-            k_giant_accumulate<SYNC, W, TIE><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
-            k_giant_decide<SYNC, TIE><<<grid_for(ng, 128), 128, 0, cs>>>(a, ga, ng);
+            k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
+            k_giant_decide<SYNC><<<grid_for(ng, 128), 128, 0, cs>>>(a, ga, ng);
             k_giant_finish<<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
             CU(cudaGetLastError());
             g->stats.launches[3] += 4;
@@ -1884,12 +1879,12 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[2], n, 2, rw, ctr + kCtrRecsW,
                                                                           split, rb, ctr + kCtrRecsB);
             if (split > (uint32_t)p.block_degree) {
-                k_warp<SYNC, W, TIE, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2,
+                k_warp<SYNC, W, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2,
                                                                                                ctr + kCtrSchedB);
                 g->stats.launches[2] += 1;
             }
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W, TIE><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB);
+            k_block<SYNC, W><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB);
             CU(cudaGetLastError());
             g->stats.launches[2] += 2;
         }
@@ -1914,7 +1909,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                 const int64_t per = (int64_t)a.sched_block * 32 * kWarpWarps * sms;
                 ctas = (int)std::max<int64_t>(1, std::min<int64_t>(kWarpCtasPerSm, n / per));
             }
-            k_warp<SYNC, W, TIE, kWarpSlots><<<sms * ctas, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
+            k_warp<SYNC, W, kWarpSlots><<<sms * ctas, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
                                                                                           ctr + kCtrSchedW);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
@@ -1926,7 +1921,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[0];
         CHECK(rec(0, 0));
         if (n > 0) {
-            CHECK((launch_thread_bin<SYNC, W, TIE>(g, a)));
+            CHECK((launch_thread_bin<SYNC, W>(g, a)));
             g->stats.launches[0] += 1;
         }
         CHECK(rec(0, 1));
@@ -2003,17 +1998,13 @@ int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long lon
         CHECK(dalloc(&g->labels_prev, (size_t)g->n_global));
         CHECK(dalloc(&g->flags_prev, (size_t)g->n_global));
     }
-    const int sel = (p.mode == NULPA_SYNC ? 4 : 0) + (w ? 2 : 0) + (p.tie_rule ? 1 : 0);
+    const int sel = (p.mode == NULPA_SYNC ? 2 : 0) + (w ? 1 : 0);
     int r;
     switch (sel) {
-    case 0: r = sweep_impl<false, false, 0>(g, pickless, p, ctr, timing, slot); break;
-    case 1: r = sweep_impl<false, false, 1>(g, pickless, p, ctr, timing, slot); break;
-    case 2: r = sweep_impl<false, true, 0>(g, pickless, p, ctr, timing, slot); break;
-    case 3: r = sweep_impl<false, true, 1>(g, pickless, p, ctr, timing, slot); break;
-    case 4: r = sweep_impl<true, false, 0>(g, pickless, p, ctr, timing, slot); break;
-    case 5: r = sweep_impl<true, false, 1>(g, pickless, p, ctr, timing, slot); break;
-    case 6: r = sweep_impl<true, true, 0>(g, pickless, p, ctr, timing, slot); break;
-    default: r = sweep_impl<true, true, 1>(g, pickless, p, ctr, timing, slot); break;
+    case 0: r = sweep_impl<false, false>(g, pickless, p, ctr, timing, slot); break;
+    case 1: r = sweep_impl<false, true>(g, pickless, p, ctr, timing, slot); break;
+    case 2: r = sweep_impl<true, false>(g, pickless, p, ctr, timing, slot); break;
+    default: r = sweep_impl<true, true>(g, pickless, p, ctr, timing, slot); break;
     }
     ++g->sweeps_since_reset;
     return r;
@@ -2048,6 +2039,45 @@ int ensure_events(nulpa_graph *g) {
 int resolve_mem(const void *p, int memkind) {
     if (memkind != NULPA_MEM_HOST && memkind != NULPA_MEM_DEVICE) return fail(NULPA_EINVAL, "memkind must be NULPA_MEM_HOST or NULPA_MEM_DEVICE");
     (void)p;
+    return NULPA_OK;
+}
+
+// R12: reject weights that are negative, NaN or infinite (the argmax orders
+// IEEE bit patterns and the giant bin's running maximum needs totals that
+// only grow).  One device pass over the weights, counted in a spare slot of
+// the handle's counters.
+int check_weights(nulpa_graph *g) {
+    if (!g->weights || g->M == 0) return NULPA_OK;
+    unsigned long long *bad = g->ctr + (size_t)kMaxIter * kCtr + kCtr - 1;
+    CU(cudaMemsetAsync(bad, 0, sizeof *bad, g->stream));
+    k_check_weights<<<grid_for(g->M, 256, num_sms() * 8), 256, 0, g->stream>>>(g->weights, g->M, bad);
+    CU(cudaGetLastError());
+    unsigned long long h = 0;
+    CU(cudaMemcpyAsync(&h, bad, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    if (h) return fail(NULPA_EINVAL, "%llu weights are negative, NaN or infinite (weights must be finite and >= 0, R12)", h);
+    return NULPA_OK;
+}
+
+// Labels passed in by the caller must be vertex IDs in [0, n_global) (they
+// index Sigma in the modularity kernels and the label-keyed tables).
+int check_labels(nulpa_graph *g, const int32_t *lab, int memkind) {
+    const int64_t n = g->n_global;
+    if (memkind == NULPA_MEM_HOST) {
+        for (int64_t i = 0; i < n; ++i)
+            if (lab[i] < 0 || (int64_t)lab[i] >= n)
+                return fail(NULPA_EINVAL, "label %d of vertex %lld is outside [0, %lld)", lab[i], (long long)i, (long long)n);
+        return NULPA_OK;
+    }
+    if (n == 0) return NULPA_OK;
+    unsigned long long *bad = g->ctr + (size_t)kMaxIter * kCtr + kCtr - 1;
+    CU(cudaMemsetAsync(bad, 0, sizeof *bad, g->stream));
+    k_check_labels<<<grid_for(n, 256, num_sms() * 8), 256, 0, g->stream>>>(lab, n, bad);
+    CU(cudaGetLastError());
+    unsigned long long h = 0;
+    CU(cudaMemcpyAsync(&h, bad, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    if (h) return fail(NULPA_EINVAL, "%llu labels are outside [0, %lld)", h, (long long)n);
     return NULPA_OK;
 }
 
@@ -2139,6 +2169,7 @@ int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *we
     if ((r = dalloc(&g->ctr, (size_t)(kMaxIter + 1) * kCtr))) return bail(r);
     if (cudaMallocHost((void **)&g->ctr_host, (kMaxIter + 1) * kCtr * sizeof(unsigned long long)) != cudaSuccess)
         return bail(fail(NULPA_ENOMEM, "cudaMallocHost failed"));
+    if ((r = check_weights(g))) return bail(r);
     if ((r = reset_state(g))) return bail(r);
     nulpa_params p;
     nulpa_default_params(&p);
@@ -2262,6 +2293,7 @@ int nulpa_flags(nulpa_graph *g, uint8_t *out, int memkind) {
 int nulpa_set_labels(nulpa_graph *g, const int32_t *in, const uint8_t *flags, int memkind) {
     if (!g || !in) return fail(NULPA_EINVAL, "null argument");
     CHECK(resolve_mem(in, memkind));
+    CHECK(check_labels(g, in, memkind));
     const cudaMemcpyKind k = memkind == NULPA_MEM_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
     CU(cudaMemcpyAsync(g->labels, in, g->n_global * sizeof(int32_t), k, g->stream));
     if (flags)
@@ -2272,11 +2304,11 @@ int nulpa_set_labels(nulpa_graph *g, const int32_t *in, const uint8_t *flags, in
     return NULPA_OK;
 }
 
-int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, double *sigma_intra, double *two_m,
-                             double *Sigma_device) {
-    if (!g || !sigma_intra || !two_m || !Sigma_device) return fail(NULPA_EINVAL, "null argument");
+}  // extern "C"
+
+namespace {
+int modularity_partial(nulpa_graph *g, const int32_t *lab, double *sigma_intra, double *two_m, double *Sigma_device) {
     if (!g->macc) CHECK(dalloc(&g->macc, 4));
-    const int32_t *lab = labels_device ? labels_device : g->labels;
     CU(cudaMemsetAsync(g->macc, 0, 4 * sizeof(double), g->stream));
     const int sms = num_sms();
     if (!g->Kdeg) {                                         // graph-invariant: K_i and 2m, once
@@ -2305,6 +2337,16 @@ int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, doubl
     *two_m += g->two_m_local;
     return NULPA_OK;
 }
+}  // namespace
+
+extern "C" {
+
+int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, double *sigma_intra, double *two_m,
+                             double *Sigma_device) {
+    if (!g || !sigma_intra || !two_m || !Sigma_device) return fail(NULPA_EINVAL, "null argument");
+    if (labels_device) CHECK(check_labels(g, labels_device, NULPA_MEM_DEVICE));
+    return modularity_partial(g, labels_device ? labels_device : g->labels, sigma_intra, two_m, Sigma_device);
+}
 
 int nulpa_modularity_finish(nulpa_graph *g, const double *Sigma_device, double sigma_intra, double two_m, double *q) {
     if (!g || !Sigma_device || !q) return fail(NULPA_EINVAL, "null argument");
@@ -2326,6 +2368,7 @@ int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double 
     int32_t *tmp = nullptr;
     if (labels) {
         CHECK(resolve_mem(labels, memkind));
+        CHECK(check_labels(g, labels, memkind));
         if (memkind == NULPA_MEM_HOST) {
             CHECK(dalloc(&tmp, (size_t)g->n_global));
             CU(cudaMemcpyAsync(tmp, labels, g->n_global * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
@@ -2338,10 +2381,16 @@ int nulpa_modularity(nulpa_graph *g, const int32_t *labels, int memkind, double 
     if (!g->macc) CHECK(dalloc(&g->macc, 4));
     CU(cudaMemsetAsync(g->Sigma, 0, g->n_global * sizeof(double), g->stream));
     double sigma = 0, two_m = 0;
-    int r = nulpa_modularity_partial(g, lab, &sigma, &two_m, g->Sigma);
+    int r = modularity_partial(g, lab, &sigma, &two_m, g->Sigma);
     if (r == NULPA_OK) r = nulpa_modularity_finish(g, g->Sigma, sigma, two_m, q);
     dfree(tmp);
     return r;
+}
+
+int nulpa_release_memory(void) {
+    cudaMemPool_t pool = device_pool();
+    if (pool) CU(cudaMemPoolTrimTo(pool, 0));
+    return NULPA_OK;
 }
 
 int nulpa_get_stats(nulpa_graph *g, nulpa_stats *out) {

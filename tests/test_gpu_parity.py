@@ -8,6 +8,9 @@ production asynchronous mode must converge, keep the per-sweep invariants
 (labels come from own/neighbour labels, Pick-Less never increases a label),
 reach modularity within 0.02 of the oracle's, and NMI >= 0.9x the oracle's.
 """
+import json
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -110,26 +113,39 @@ def test_sync_sweep_from_random_state(gname, pickless):
 # synchronous mode, weighted: label-for-label except float32 near-ties
 # ---------------------------------------------------------------------------
 
-def near_tie(w1, w2, deg):
-    """Top-two label weights too close for two float32 summation orders to
-    agree on: within 1e-5 relative (north star) or within the worst-case
-    recursive-summation error of two float32 sums of `deg` positive terms
-    (2 * deg * 2^-24 relative, Higham 2002 eq. 4.4)."""
+NEAR_TIE_REL = 1e-5      # north star: a weighted sync label may differ only here
+
+
+def near_tie(w1, w2):
+    """The oracle's top-two label weights are within 1e-5 relative (north
+    star), so two float32 summation orders may pick either label."""
     w1 = np.asarray(w1, np.float64)
     w2 = np.asarray(w2, np.float64)
-    gap = w1 - w2
-    tol = np.maximum(1e-5, 2.0 * np.asarray(deg, np.float64) * 2.0 ** -24) * np.abs(w1)
-    return (w2 >= 0) & (gap <= tol)
+    return (w2 >= 0) & (w1 - w2 <= NEAR_TIE_REL * np.abs(w1))
+
+
+def neighbourhood(h, verts):
+    """Vertices adjacent to any of `verts` (their flags depend on whether
+    `verts` moved)."""
+    off, idx = h.offsets, h.indices
+    out = [idx[off[i]:off[i + 1]] for i in verts]
+    return np.unique(np.concatenate(out)) if out else np.zeros(0, np.int64)
+
+
+EXEMPTIONS = {}          # (graph, bins) -> labels that differed at a near-tie (reported by the test)
 
 
 @pytest.mark.parametrize("gname", ["sbm", "web", "hub", "rmat", "road", "cliques"])
 @pytest.mark.parametrize("bins", ["default", "mixed", "giant"])
 def test_sync_weighted_stepwise(gname, bins):
     """Every sweep of a full synchronous run, GPU vs oracle from the same
-    state (the oracle's; the GPU is re-seeded with it after each sweep)."""
+    state (the oracle's; the GPU is re-seeded with it after each sweep).
+    Labels must match except where the oracle's top-two label weights are
+    within 1e-5 relative (north star); flags must match outside the
+    neighbourhoods of such vertices; dN differs by at most the number of
+    exempt vertices."""
     g = GRAPHS[gname](True)
     h = host(g)
-    deg = np.diff(h.offsets)
     gg = to_gpu(g)
     C = np.arange(g.N, dtype=np.int32)
     U = np.ones(g.N, dtype=np.uint8)
@@ -140,16 +156,21 @@ def test_sync_weighted_stepwise(gname, bins):
         gg.set_labels(torch.from_numpy(C).cuda(), torch.from_numpy(U).cuda())
         gdn = gg.sweep(pl, mode=nl.SYNC, **BINS[bins])
         gC = gg.labels(device=False).numpy()
+        gU = gg.flags(device=False).numpy()
         diff = np.nonzero(gC != C1)[0]
         if diff.size:
-            ok = near_tie(w1[diff], w2[diff], deg[diff])
-            assert ok.all(), f"sweep {l}: {diff[~ok][:10]} differ without a near-tie"
+            ok = near_tie(w1[diff], w2[diff])
+            assert ok.all(), f"sweep {l}: {diff[~ok][:10]} differ without a 1e-5 near-tie"
             total_exempt += diff.size
+        fdiff = np.nonzero(gU != U1)[0]
+        if fdiff.size:
+            assert np.isin(fdiff, neighbourhood(h, diff)).all(), f"sweep {l}: flags differ at {fdiff[:10]}"
         assert abs(gdn - dn) <= diff.size
         C, U = C1, U1
         if not pl and dn / g.N < 0.05:
             break
-    assert total_exempt <= max(5, g.N // 1000)
+    EXEMPTIONS[(gname, bins)] = total_exempt
+    print(f"[weighted sync] {gname}/{bins}: {total_exempt} near-tie exemptions (1e-5 relative)")
 
 
 # ---------------------------------------------------------------------------
@@ -188,17 +209,13 @@ def test_async_sweep_invariants(gname, bins):
 @pytest.mark.parametrize("gname", ["sbm", "web", "rmat", "road", "kmer", "hub"])
 @pytest.mark.parametrize("weighted", [False, True])
 def test_async_quality_vs_oracle(gname, weighted):
-    """North star: async modularity within 0.02 of the oracle's.  The GPU's
-    schedule lies between the oracle's two schedules -- Gauss-Seidel in ID
-    order (async) and Jacobi (sync); on a graph this small one sweep is a
-    single wave, i.e. nearly Jacobi -- so the reference is the lower of the
-    two oracle runs (on k-mer paths the sequential sweep reaches 0.953, the
-    synchronous one 0.936, the GPU 0.934)."""
+    """North star: the asynchronous run converges, its modularity is within
+    0.02 of the asynchronous oracle's (Algorithm 1, sequential in-place
+    sweep), and NMI against the planted partition >= 0.9x the oracle's."""
     g = GRAPHS[gname](weighted)
     h = host(g)
     C_o, it_o, _ = oracle.lpa(h)
-    C_s, _, _ = oracle.lpa(h, sync=True)
-    q_o = min(oracle.modularity(h, C_o), oracle.modularity(h, C_s))
+    q_o = oracle.modularity(h, C_o)
     gg = to_gpu(g)
     st = gg.run()
     C_g = gg.labels(device=False).numpy()
@@ -294,6 +311,35 @@ def test_host_memkind_create_matches_device():
     assert torch.equal(a.labels(), b.labels())
 
 
+def test_input_validation():
+    """R12: weights must be finite and >= 0; labels handed in must be vertex IDs."""
+    g = synth.sbm(n=2000, community_size=50, avg_degree=8, mu=0.2, seed=3, weighted=True)
+    for bad in (-0.5, float("nan"), float("inf")):
+        w = g.weights.clone()
+        w[17] = bad
+        with pytest.raises(nl.NulpaError):
+            nl.Graph(g.offsets.cuda(), g.indices.cuda(), w.cuda())
+        with pytest.raises(nl.NulpaError):
+            nl.Graph(g.offsets, g.indices, w)                  # host memkind: checked after the copy
+    gg = to_gpu(g)
+    lab = torch.arange(g.N, dtype=torch.int32)
+    for v in (-1, g.N):
+        bad = lab.clone()
+        bad[5] = v
+        with pytest.raises(nl.NulpaError):
+            gg.set_labels(bad.cuda())
+        with pytest.raises(nl.NulpaError):
+            gg.set_labels(bad)
+        with pytest.raises(nl.NulpaError):
+            gg.modularity(bad.cuda())
+        with pytest.raises(nl.NulpaError):
+            gg.modularity(bad)
+    # a rejected set_labels leaves the state alone
+    assert torch.equal(gg.labels(device=False), lab)
+    gg.set_labels(lab.cuda())
+    assert abs(gg.modularity() - oracle.modularity(host(g), lab.numpy())) < 1e-9
+
+
 def test_invalid_params_raise():
     gg = to_gpu(synth.karate())
     with pytest.raises(nl.NulpaError):
@@ -308,6 +354,8 @@ def test_invalid_params_raise():
         gg.run(first_sweep_block=0)
     with pytest.raises(nl.NulpaError):
         gg.run(sweep_block=2000)
+    with pytest.raises(nl.NulpaError):
+        gg.run(tie_rule=1)
 
 
 # warp-bin schedules: (first_sweep_block, sweep_block); 3 and 5 leave ragged
@@ -335,7 +383,7 @@ def test_sync_schedule_independent(gname, sched):
 def test_async_schedule_invariants_and_quality(gname, sched):
     """Asynchronous runs under every schedule: dN = changed labels, labels
     from own/neighbour labels, Pick-Less never increases a label, and
-    modularity within 0.02 of the lower of the oracle's two schedules."""
+    modularity within 0.02 of the asynchronous oracle's."""
     g = GRAPHS[gname](False)
     h = host(g)
     gg = to_gpu(g)
@@ -350,8 +398,7 @@ def test_async_schedule_invariants_and_quality(gname, sched):
         check_async_sweep(h, C, C2, pl)
         C = C2
     C_o, _, _ = oracle.lpa(h)
-    C_s, _, _ = oracle.lpa(h, sync=True)
-    q_o = min(oracle.modularity(h, C_o), oracle.modularity(h, C_s))
+    q_o = oracle.modularity(h, C_o)
     gg.run(**kw)
     assert oracle.modularity(h, gg.labels(device=False).numpy()) >= q_o - 0.02
 
@@ -408,21 +455,6 @@ def test_shards_sync_equal_oracle(gname, world):
     assert abs(q - oracle.modularity(host(g), C)) < 1e-9
 
 
-# ---------------------------------------------------------------------------
-# tie rule 1 (R6 alternative: first in slot order = smallest k mod p1, then k)
-# ---------------------------------------------------------------------------
-
-@pytest.mark.parametrize("gname", ["karate", "sbm", "web", "hub", "road"])
-@pytest.mark.parametrize("bins", ["default", "mixed", "block", "giant"])
-def test_sync_tie_slot_bit_exact(gname, bins):
-    g = GRAPHS[gname](False)
-    C, it, dn = oracle.lpa(host(g), sync=True, tie_rule=1)
-    gg = to_gpu(g)
-    st = gg.run(mode=nl.SYNC, tie_rule=nl.TIE_SLOT, **BINS[bins])
-    assert st["iterations"] == it and st["changed"] == list(dn)
-    np.testing.assert_array_equal(gg.labels(device=False).numpy(), C)
-
-
 def test_distributed_driver_nccl_world1():
     """The real multi-GPU driver (Exchanger: NCCL all-gather of labels,
     reduce-scatter(MAX) of flags, all-reduce of dN) on a one-rank NCCL group:
@@ -449,8 +481,7 @@ def test_distributed_driver_nccl_world1():
         res = D.lpa_distributed(runner_a)
         assert res["converged"]
         C_o, _, _ = oracle.lpa(h)
-        C_s, _, _ = oracle.lpa(h, sync=True)
-        q_o = min(oracle.modularity(h, C_o), oracle.modularity(h, C_s))
+        q_o = oracle.modularity(h, C_o)
         assert oracle.modularity(h, runner_a.labels.cpu().numpy()) >= q_o - 0.02
         assert abs(D.modularity_distributed(runner_a) - oracle.modularity(h, runner_a.labels.cpu().numpy())) < 1e-9
     finally:
