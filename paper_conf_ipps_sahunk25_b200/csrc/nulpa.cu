@@ -323,8 +323,6 @@ struct SweepArgs {
     uint8_t *flag_out;
     int64_t row_begin;
     int pickless;
-    int sched_block;           // warp-bin schedule: record groups per block (k_warp)
-    int split;                 // 1: warp-bin k_warp takes one contiguous 1/nw of the groups per warp
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 
@@ -430,32 +428,70 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
 // p1 in {255, 511} (a Mersenne number as in R1/R3, load factor <= 1/4 for
 // D < 64 and <= 1/2 above; PAPER.md:208 sizes per-vertex GLOBAL tables
 // p1 = nextPow2(D)-1 -- the giant bin keeps that sizing).  One 64-bit word
-// per slot (key | float value), so a probe is ONE ld.shared.b64; the table
-// is cleared with 16-byte stores before each vertex (hashtableClear,
-// PAPER.md:333).  Keys within one 32-entry batch are distinct (one leader per
-// label, match_any), batches are ordered by __syncwarp, so the value update
-// is a plain read-modify-write; only the slot claim is atomic.
+// per slot {tag k+1, float value}, so a probe is ONE ld.shared.v2 and an
+// empty slot is all-zero (its value 0.0f, so "claim" and "hit" both store
+// old value + x); the table is cleared with 16-byte stores of the zero
+// register before each vertex (hashtableClear).  Keys within
+// one 32-entry batch are distinct (one leader per label, match_any) and
+// batches are ordered by __syncwarp, so the value update is a plain
+// read-modify-write; only the slot claim is atomic.
 // ---------------------------------------------------------------------------
 constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 
-// Algorithm 2's probe sequence past the home slot (hybrid quadratic-double
-// probing, R5 linear continuation) on a one-word-per-slot table of capacity P.
-// Continues after probe t0 at slot i (t0 = 0: the home slot; t0 = 1: home + 1,
-// where the step delta_1 = 1 has become delta_2 = 2 + (k mod p2) mod P).
-#ifndef NULPA_PROBE2
-#define NULPA_PROBE2 1
-#endif
+// Slot claims without atomics.  A full-warp shared-memory atomic costs ~2
+// cycles per active lane of the SM's atomics unit (B300_MICROARCH.md
+// "Atomics"), and in the first sweep ~25 leaders per batch claim new slots,
+// so the claim is a warp-synchronous round instead: every probing lane
+// reads its slot (one ld.shared.v2 per lane), lanes that find their tag are
+// done (hit), lanes that find it empty store their tag, __syncwarp, and
+// re-read it -- of several lanes storing to one slot in the same round
+// exactly one store survives, that lane won the claim, the others probe on.
+// The value update is old value + x (an empty slot holds 0.0f), stored by
+// the lane that owns the label's slot.  `need` lanes probe; on return they
+// are done (need = false) or collided.
+__device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, float x, bool &need, float &V) {
+    uint32_t n = need, vb = __float_as_uint(V);
+    asm volatile(
+        "{\n\t"
+        ".reg .pred pn, ph, pc, pd;\n\t"
+        ".reg .b32 ck, now;\n\t"
+        ".reg .f32 cv, nv;\n\t"
+        "setp.ne.b32 pn, %0, 0;\n\t"
+        "mov.b32 ck, 0xFFFFFFFF;\n\t"
+        "mov.f32 cv, 0f00000000;\n\t"
+        "@pn ld.shared.v2.b32 {ck, cv}, [%2];\n\t"
+        "setp.eq.b32 ph, ck, %3;\n\t"              // the label's slot: hit
+        "setp.eq.b32 pc, ck, 0;\n\t"               // empty: try to claim
+        "@pc st.shared.b32 [%2], %3;\n\t"
+        "bar.warp.sync 0xFFFFFFFF;\n\t"
+        "mov.b32 now, 0;\n\t"
+        "@pc ld.shared.b32 now, [%2];\n\t"
+        "setp.eq.and.b32 pd, now, %3, pc;\n\t"     // this lane's store survived: claimed
+        "or.pred pd, pd, ph;\n\t"
+        "add.rn.f32 nv, cv, %4;\n\t"
+        "@pd st.shared.f32 [%2+4], nv;\n\t"
+        "@pd mov.b32 %1, nv;\n\t"
+        "@pd mov.b32 %0, 0;\n\t"
+        "}"
+        : "+r"(n), "+r"(vb)
+        : "r"(addr), "r"(tg), "f"(x)
+        : "memory");
+    need = n != 0;
+    V = __uint_as_float(vb);
+}
+
+// Algorithm 2's probe sequence past probe 1 (home + 1; the step delta_0 = 1
+// has become delta_1 = 2 + (k mod p2) mod P): hybrid quadratic-double
+// probing, R5 linear continuation after kMaxRetries probes.  Called by the
+// whole warp (rounds are warp-synchronous); lanes without `need` idle.
 template <uint32_t P>
-__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint32_t i, int t0) {
+__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint32_t i, bool need, float V) {
     constexpr uint32_t p2 = 2 * P + 1;                    // R3
     const uint32_t km = ((uint32_t)k % p2) % P;
-    uint32_t di = 1;
-    if (t0 == 1) {
-        di = 2 + km;
-        if (di >= P) di -= P;
-    }
+    uint32_t di = 2 + km;
+    if (di >= P) di -= P;
     const uint32_t tg = kv_tag(k);
-    for (int t = t0 + 1;; ++t) {
+    for (int t = 2; __any_sync(0xFFFFFFFFu, need); ++t) {
         if (t <= kMaxRetries) {
             i += di;
             if (i >= P) i -= P;
@@ -465,58 +501,28 @@ __device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint
         } else {
             i = i + 1 == P ? 0 : i + 1;                    // R5
         }
-        const uint64_t cur = lds_u64(tab + 8 * i);
-        const uint32_t ck = (uint32_t)cur;
-        if (ck == tg) {
-            const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
-            sts_f32(tab + 8 * i + 4, V);
-            return V;
-        }
-        if (ck == kTagEmpty && cas_u32(tab + 8 * i, kTagEmpty, tg) == kTagEmpty) {
-            sts_f32(tab + 8 * i + 4, x);
-            return x;
-        }
+        kv_round(tab + 8 * i, tg, x, need, V);
     }
+    return V;
 }
 
-// hashtableAccumulate (Algorithm 2) for a leader adding its group's weight x
-// to label k; keys of one batch are distinct, so only the claim is atomic.
-// Returns the label's new total.
+// hashtableAccumulate (Algorithm 2) by the group leaders of one batch (`on`),
+// adding group weight x to label k: the home slot k mod P and probe 1
+// (home + 1) inline, later probes out of line.  Returns the label's new
+// total (leaders only).  Warp-synchronous: called by all 32 lanes.
 template <uint32_t P>
-__device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, float x) {
-    const uint32_t i = (uint32_t)k % P;
+__device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, float x, bool on) {
     const uint32_t tg = kv_tag(k);
-    const uint64_t cur = lds_u64(tab + 8 * i);
-    const uint32_t ck = (uint32_t)cur;
-    if (ck == tg) {
-        const float V = __fadd_rn(__uint_as_float((uint32_t)(cur >> 32)), x);
-        sts_f32(tab + 8 * i + 4, V);
-        return V;
+    const uint32_t i0 = (uint32_t)k % P;
+    float V = 0.0f;
+    bool need = on;
+    kv_round(tab + 8 * i0, tg, x, need, V);
+    if (__any_sync(0xFFFFFFFFu, need)) {
+        const uint32_t i1 = i0 + 1 == P ? 0u : i0 + 1;
+        kv_round(tab + 8 * i1, tg, x, need, V);
+        if (__any_sync(0xFFFFFFFFu, need)) V = kv_add_slow<P>(tab, k, x, i1, need, V);
     }
-    if (ck == kTagEmpty && cas_u32(tab + 8 * i, kTagEmpty, tg) == kTagEmpty) {
-        sts_f32(tab + 8 * i + 4, x);
-        return x;
-    }
-#if NULPA_PROBE2
-    // Probe 1 of the sequence (delta_0 = 1: the next slot) inline: with ~25
-    // leaders per batch some lane almost always collides at home in the first
-    // sweep, and the warp would take the out-of-line path together.
-    const uint32_t i1 = i + 1 == P ? 0u : i + 1;
-    const uint64_t cur1 = lds_u64(tab + 8 * i1);
-    const uint32_t ck1 = (uint32_t)cur1;
-    if (ck1 == tg) {
-        const float V = __fadd_rn(__uint_as_float((uint32_t)(cur1 >> 32)), x);
-        sts_f32(tab + 8 * i1 + 4, V);
-        return V;
-    }
-    if (ck1 == kTagEmpty && cas_u32(tab + 8 * i1, kTagEmpty, tg) == kTagEmpty) {
-        sts_f32(tab + 8 * i1 + 4, x);
-        return x;
-    }
-    return kv_add_slow<P>(tab, k, x, i1, 1);
-#else
-    return kv_add_slow<P>(tab, k, x, i, 0);
-#endif
+    return V;
 }
 
 // ---------------------------------------------------------------------------
@@ -630,51 +636,47 @@ __global__ void __launch_bounds__(kFrontThreads) k_frontier(SweepArgs a, const i
 }
 
 // ---------------------------------------------------------------------------
-// warp-per-vertex kernel (switch_degree <= D < block_degree), over the
-// compacted frontier and software-pipelined across the vertices of a warp.
-// A warp owns record groups gw, gw + nw, ... (32 records each) and walks them
-// as one sequence n = 0, 1, ...; while vertex n is folded, the label gathers
-// of vertex n+1 and the index/weight loads of vertex n+2 are in flight, so
-// each dependent global round trip overlaps a whole vertex of work.  Records
-// reach shared memory one group ahead (a 2-group ring per warp).
+// warp-per-vertex kernel (switch_degree <= D < block_degree; the wide variant
+// serves the block bin below wide_degree), over the compacted frontier and
+// software-pipelined across the vertices of a warp.  A warp walks its record
+// groups (32 records each; 4 in the wide variant) as one sequence
+// n = 0, 1, ...; while vertex n is folded, the label gathers of vertex n+1
+// and the index/weight loads of vertex n+2 are in flight, so each dependent
+// global round trip overlaps a whole vertex of work.  Records reach shared
+// memory one group ahead (a 2-group ring per warp).
 // Per 32-entry batch: match_any folds lanes holding the same label onto a
-// leader, whose group total (count * w when the batch's weights are all
+// leader, whose group total (count * w when the vertex's weights are all
 // equal, else a pairwise tree) is added into the table (Algorithm 2); each
-// lane keeps the best (total, label) it produced as a leader, and two
-// redux.max give hashtableMaxKey without scanning the table.  Degree <= 32
-// needs no table (the match groups are the totals).
+// lane keeps the best (total, label) it produced as a leader, and a
+// redux.max / redux.min pair gives hashtableMaxKey without scanning the
+// table (ties: smallest label, R6).  Degree <= 32 needs no table (the match
+// groups are the totals).
 // Asynchronous reading: vertex n+1's neighbour labels are gathered before
 // vertex n's new label is written; the gathered copies of that label are
 // patched in registers, so n+1 still sees n's move.
+//
+// Which record groups a warp walks (WarpSched):
+//  * SCHED_STEAL (first sweep after a reset): warp w owns the contiguous
+//    groups [w*ng/nw, (w+1)*ng/nw) -- one long run of consecutive rows, so
+//    labels propagate along ID order as in the sequential Algorithm 1
+//    (modularity) -- and a warp that runs dry
+//    steals the far half of the remaining range of the most-loaded of 32
+//    sampled warps (the victim's run continues undisturbed; the tail is
+//    balanced).  A range is one 64-bit word {next group, end group}: the
+//    owner takes a group with atomicAdd on the low half, a thief shrinks
+//    the high half with atomicCAS.
+//  * SCHED_GUIDED (K > 1): guided chunks of min(K, groups left / nw)
+//    consecutive groups from a global counter.
+//  * SCHED_STRIDED (K = 1): groups w, w + nw, ...
 // ---------------------------------------------------------------------------
 constexpr int kWarpWarps = 8;            // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
-#ifndef NULPA_GUIDED_C
-#define NULPA_GUIDED_C 1                 // guided chunk = min(K, groups left / (C * warps)) ...
-#endif
-#ifndef NULPA_FIRST_SPLIT
-#define NULPA_FIRST_SPLIT 0              // first sweep: contiguous equal split of the warp-bin groups
-#endif
-#ifndef NULPA_GUIDED_DIV
-#define NULPA_GUIDED_DIV 4               // ... but at least K / this (0: min(K, NULPA_GUIDED_MIN)): the
-                                         // first sweep's chunks (K = 128) never drop below 32 groups
-                                         // (DESIGN.md "Quality notes"); later sweeps (K = 4) keep 1
-#endif
-#ifndef NULPA_GUIDED_MIN
-#define NULPA_GUIDED_MIN 1
-#endif
-
-constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM: 64 registers per thread
-// The wide variant (block-bin vertices below wide_degree <= 512): 1024-slot
+constexpr int kWarpCtasPerSm = NULPA_WARP_CTAS;   // 32 warps/SM
+// The wide variant (block-bin vertices below wide_degree <= 1024): 1024-slot
 // tables (8 KB per warp, p1 = 1023), 4 warps per CTA, 6 CTAs (24 warps) per SM.
 constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
-// Records per group (the unit a warp takes from the frontier): 32 in the warp
-// bin; the wide variant takes groups of NULPA_WIDE_GROUP (4) records from a
-// dynamic counter -- its ~200K vertices of degree 256..511 in 32-record groups
-// were only ~1.8 groups per warp, and the static strided split left half the
-// warps idle for the second half of the launch.
 #ifndef NULPA_WIDE_GROUP
 #define NULPA_WIDE_GROUP 4
 #endif
@@ -684,229 +686,304 @@ constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
 template <int SLOTS> struct WarpCfg {
     static constexpr int warps = SLOTS == kWarpSlots ? kWarpWarps : kWideWarps;
     static constexpr int ctas = SLOTS == kWarpSlots ? kWarpCtasPerSm : kWideCtasPerSm;
-    static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step
+    static constexpr int unroll = SLOTS == kWarpSlots ? 2 : 4;   // 32-entry batches per loop step past 64
     static constexpr int group = SLOTS == kWarpSlots ? 32 : NULPA_WIDE_GROUP;
+};
+
+enum { SCHED_STRIDED = 0, SCHED_GUIDED = 1, SCHED_STEAL = 2 };
+#ifndef NULPA_MIN_RUN
+#define NULPA_MIN_RUN 2048
+#endif
+constexpr int64_t kMinFirstRun = NULPA_MIN_RUN;   // rows per warp in the first sweep, at least (small bins)
+struct WarpSched {
+    int mode;
+    int K;                               // guided chunk size (groups)
+    unsigned long long *counter;         // guided: next group
+    unsigned long long *ranges;          // steal: one {next, end} word per warp
+};
+
+// The warp's next record group, or 0xFFFFFFFF once the warp's share of the
+// frontier is exhausted (sticky).  Warp-uniform.
+struct GroupFetcher {
+    uint32_t cur, lim;                   // strided: next group; guided: chunk [cur, lim)
+    uint32_t ng, nw, gw;
+    bool dry;
+    __device__ __forceinline__ uint32_t next(const WarpSched &s, int lane) {
+        if (dry) return 0xFFFFFFFFu;
+        uint32_t g = 0xFFFFFFFFu;
+        if (s.mode == SCHED_STRIDED) {
+            if (cur < ng) g = cur;
+            cur += nw;
+        } else if (s.mode == SCHED_GUIDED) {
+            if (cur >= lim) {
+                uint32_t start = 0, size = 1;
+                if (lane == 0) {
+                    const uint32_t done = (uint32_t)min((unsigned long long)ng, *(volatile unsigned long long *)s.counter);
+                    size = max(1u, min((uint32_t)s.K, (ng - done) / nw));
+                    start = (uint32_t)min((unsigned long long)ng, atomicAdd(s.counter, (unsigned long long)size));
+                }
+                cur = __shfl_sync(0xFFFFFFFFu, start, 0);
+                lim = min(ng, cur + __shfl_sync(0xFFFFFFFFu, size, 0));
+            }
+            if (cur < lim) g = cur++;
+        } else {                                           // SCHED_STEAL
+            for (;;) {
+                if (lane == 0) {
+                    const unsigned long long w = atomicAdd(s.ranges + gw, 1ull);   // next group of the own range
+                    g = (uint32_t)w < (uint32_t)(w >> 32) ? (uint32_t)w : 0xFFFFFFFFu;
+                }
+                g = __shfl_sync(0xFFFFFFFFu, g, 0);
+                if (g != 0xFFFFFFFFu || !steal(s, lane)) break;
+            }
+        }
+        dry = g == 0xFFFFFFFFu;
+        return g;
+    }
+    // Sample 32 warps per round (one per lane), pick the one with the most
+    // groups left and move the far half of its range into the own word.
+    // false after 8 rounds without a warp holding >= 2 groups.
+    __device__ __noinline__ bool steal(const WarpSched &s, int lane) {
+        int fails = 0;
+        for (uint32_t round = 0; round < 8;) {
+            uint32_t h = (gw * 0x9E3779B9u) ^ ((round * 32u + (uint32_t)lane + 1u) * 0x85EBCA6Bu);
+            h ^= h >> 15;
+            h *= 0x2C1B3C6Du;
+            h ^= h >> 12;
+            const uint32_t v = h % nw;
+            unsigned long long w = 0;
+            int32_t rem = 0;
+            if (v != gw) {
+                w = *(volatile unsigned long long *)(s.ranges + v);
+                rem = (int32_t)((uint32_t)(w >> 32) - (uint32_t)w);
+            }
+            const int32_t best = __reduce_max_sync(0xFFFFFFFFu, rem);
+            if (best < 2) {
+                ++round;
+                continue;
+            }
+            const int src = __ffs(__ballot_sync(0xFFFFFFFFu, rem == best)) - 1;
+            uint32_t ok = 0;
+            if (lane == src) {
+                const uint32_t lo = (uint32_t)w, hi = (uint32_t)(w >> 32);
+                const uint32_t mid = hi - (uint32_t)rem / 2;           // victim keeps [lo, mid)
+                if (atomicCAS(s.ranges + v, w, ((unsigned long long)mid << 32) | lo) == w) {
+                    atomicExch(s.ranges + gw, ((unsigned long long)hi << 32) | mid);
+                    ok = 1;
+                }
+            }
+            if (__shfl_sync(0xFFFFFFFFu, ok, src)) return true;
+            if (++fails > 32) return false;                // lost races: try the same round again
+        }
+        return false;
+    }
 };
 
 template <bool SYNC, bool W, int SLOTS>
 __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ctas)
     k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin,
-           unsigned long long *sched) {
-    constexpr int kWarpWarps = WarpCfg<SLOTS>::warps;
+           WarpSched ws) {
+    constexpr int NWARP = WarpCfg<SLOTS>::warps;
     constexpr int U = WarpCfg<SLOTS>::unroll;
     constexpr int G = WarpCfg<SLOTS>::group;
+    constexpr uint32_t RING = 2 * G;
     static_assert(G >= 1 && G <= 32 && (G & (G - 1)) == 0, "group size: power of two <= 32");
-    __shared__ __align__(16) uint64_t s_tab[kWarpWarps][SLOTS];
-    __shared__ VRec s_ring[kWarpWarps][2 * G];        // two groups; record m sits at m mod 2G
+    __shared__ __align__(16) uint64_t s_tab[NWARP][SLOTS];
+    __shared__ __align__(16) VRec s_ring[NWARP][RING];   // two groups; record m sits at m mod 2G
     __shared__ unsigned long long bctr[2];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const uint32_t tab = (uint32_t)__cvta_generic_to_shared(&s_tab[wid][0]);
+    const uint32_t ring = (uint32_t)__cvta_generic_to_shared(&s_ring[wid][0]);
+    const unsigned lanes_below = (1u << lane) - 1;
     if (threadIdx.x < 2) bctr[threadIdx.x] = 0;
-    __syncthreads();
-    const int64_t nrec = (int64_t)*count;
-    const int64_t nw = (int64_t)gridDim.x * kWarpWarps;
-    const int64_t gw = (int64_t)blockIdx.x * kWarpWarps + wid;
-    const int64_t ng = (nrec + G - 1) / G;
-    // Record groups of this warp.  K = 1: static strided, groups gw, gw + nw, ...
-    // K > 1: dynamic (guided) chunks -- a warp grabs its next chunk of
-    // min(K, groups left / nw) consecutive groups from a global counter, so
-    // it walks runs of up to 32K consecutive rows in order (labels propagate
-    // along ID order as in the sequential Algorithm 1: modularity) and the
-    // chunks shrink toward the end of the sweep.  (A static K-block schedule
-    // gave each warp only ~2 blocks per sweep and left a long tail.)
-    const int64_t K = SLOTS == kWarpSlots ? a.sched_block : NULPA_WIDE_K;
-    // split (first sweep, NULPA_FIRST_SPLIT): warp gw walks the contiguous
-    // groups [gw * ng / nw, (gw + 1) * ng / nw) -- one run per warp, the fewest
-    // run starts, no tail from chunk granularity
-    const bool split = SLOTS == kWarpSlots && a.split;
-    const bool dyn = K > 1 && !split;
-    int64_t cur = dyn ? 0 : gw, lim = dyn ? 0 : ng;        // static: next group cur (step nw); dynamic: chunk [cur, lim)
-    if (split) {
-        cur = gw * ng / nw;
-        lim = (gw + 1) * ng / nw;
+    const uint32_t nrec = (uint32_t)*count;
+    GroupFetcher F;
+    F.ng = (nrec + G - 1) / G;
+    F.nw = gridDim.x * NWARP;
+    F.gw = blockIdx.x * NWARP + wid;
+    F.cur = ws.mode == SCHED_STRIDED ? F.gw : 0;
+    F.lim = 0;
+    F.dry = false;
+    if (ws.mode == SCHED_STEAL && lane == 0) {
+        // initial ranges of >= K groups each (K = kMinFirstRun / 32: long runs
+        // on small bins); warps past ng / K start empty and only steal
+        const uint32_t nr = max(1u, min(F.nw, F.ng / max(1, ws.K)));
+        const uint32_t b = F.gw < nr ? (uint32_t)((uint64_t)F.gw * F.ng / nr) : 0u;
+        const uint32_t e = F.gw < nr ? (uint32_t)((uint64_t)(F.gw + 1) * F.ng / nr) : 0u;
+        atomicExch(ws.ranges + F.gw, ((unsigned long long)e << 32) | b);
     }
-    const int64_t stride = dyn || split ? 1 : nw;
-    unsigned long long c_ch = 0, c_che = 0;
-    auto grec_next = [&]() -> VRec {                       // lane's record of the warp's next group (or empty)
-        VRec z{0, 0, 0, 0};
-        if (dyn && cur >= lim) {
-            unsigned long long start = 0, size = 1;
-            if (lane == 0) {
-                const int64_t left = ng - (int64_t)*(volatile unsigned long long *)sched;
-#if NULPA_GUIDED_DIV
-                const int64_t floor_k = std::max<int64_t>(1, K / NULPA_GUIDED_DIV);
-#else
-                const int64_t floor_k = std::min<int64_t>(K, NULPA_GUIDED_MIN);
-#endif
-                size = (unsigned long long)std::max<int64_t>(floor_k, std::min<int64_t>(K, left / (NULPA_GUIDED_C * nw)));
-                start = atomicAdd(sched, size);
-            }
-            cur = (int64_t)__shfl_sync(0xFFFFFFFFu, start, 0);
-            lim = std::min<int64_t>(ng, cur + (int64_t)__shfl_sync(0xFFFFFFFFu, size, 0));
-        }
-        if (cur >= lim) return z;
-        const int64_t i = cur * G + lane;
-        cur += stride;
-        return lane < G && i < nrec ? recs[i] : z;
+    __syncthreads();
+    // lane's record of group g.  Past the warp's last group: end records
+    // (r = -1); past the bin inside the bin's last group: degree-0 no-op
+    // records (with work stealing the bin's last group need not be the
+    // warp's last)
+    auto grec = [&](uint32_t g) -> VRec {
+        if (g == 0xFFFFFFFFu || lane >= G) return VRec{0, 0, -1, 0};
+        const uint32_t i = g * G + lane;
+        return i < nrec ? recs[i] : VRec{0, 0, 0, 0};
     };
-    auto rrec = [&](int m) -> VRec { return s_ring[wid][m & (2 * G - 1)]; };
+    auto rrec = [&](uint32_t m) -> VRec {
+        VRec r;
+        asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(r.o_lo), "=r"(r.o_hi_deg), "=r"(r.r), "=r"(r.ci)
+                     : "r"(ring + 16u * (m & (RING - 1))) : "memory");
+        return r;
+    };
     auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
     {
-        const VRec r0 = grec_next(), r1 = grec_next();   // zero records (degree 0) past the end
+        const VRec r0 = grec(F.next(ws, lane));
+        const VRec r1 = grec(F.next(ws, lane));
         if (lane < G) {
             s_ring[wid][lane] = r0;
             s_ring[wid][G + lane] = r1;
         }
     }
-    VRec pend = grec_next();
+    VRec pend = grec(F.next(ws, lane));
     __syncwarp();
-    // pipeline registers of one vertex: entries lane and lane+32 of its row
-    // (index j, weight w, neighbour label k)
-    struct Stage {
-        int32_t ja, jb;
-        float wa, wb;
-        int32_t ka, kb;
-    };
-    Stage SA{-1, -1, 1.0f, 1.0f, kEmpty, kEmpty}, SB = SA, SC = SA;
-    auto load_row = [&](int m, int32_t &ja, int32_t &jb, float &wa, float &wb) {
-        ja = jb = -1;
+    const int32_t *__restrict__ lab_in = a.lab_in;
+    // row loads: entries lane and lane+32 of the row of record m
+    auto load_row = [&](const VRec &r, int32_t &ja, int32_t &jb, float &wa, float &wb) {
+        const uint32_t d = r_d(r);
+        const int64_t o = r_o(r);
+        const int32_t *pi = a.indices + o + lane;
+        ja = (uint32_t)lane < d ? ld_stream(pi) : -1;
+        jb = (uint32_t)lane + 32 < d ? ld_stream(pi + 32) : -1;
         wa = wb = 1.0f;
-        {   // past the end the ring holds zero records (degree 0): no loads
-            const VRec r = rrec(m);
-            const uint32_t d = r_d(r);
-            const int64_t o = r_o(r);
-            if ((uint32_t)lane < d) ja = ld_stream(a.indices + o + lane);
-            if ((uint32_t)lane + 32 < d) jb = ld_stream(a.indices + o + 32 + lane);
-            if (W) {
-                if ((uint32_t)lane < d) wa = ld_stream(a.weights + o + lane);
-                if ((uint32_t)lane + 32 < d) wb = ld_stream(a.weights + o + 32 + lane);
-            }
+        if (W) {
+            const float *pw = a.weights + o + lane;
+            if ((uint32_t)lane < d) wa = ld_stream(pw);
+            if ((uint32_t)lane + 32 < d) wb = ld_stream(pw + 32);
         }
     };
-    auto gather = [&](int m, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
-        ka = kb = kEmpty;
-        {
-            const int32_t vk = (int32_t)(rrec(m).r + a.row_begin);
-            if (ja >= 0 && ja != vk) ka = a.lab_in[ja];     // "if j = i continue"
-            if (jb >= 0 && jb != vk) kb = a.lab_in[jb];
-        }
+    // label gathers ("if j = i continue": the vertex's own entries are skipped)
+    auto gather = [&](int32_t vk, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
+        ka = (ja >= 0 && ja != vk) ? lab_in[ja] : kEmpty;
+        kb = (jb >= 0 && jb != vk) ? lab_in[jb] : kEmpty;
     };
-    load_row(0, SA.ja, SA.jb, SA.wa, SA.wb);
-    load_row(1, SB.ja, SB.jb, SB.wa, SB.wb);
-    gather(0, SA.ja, SA.jb, SA.ka, SA.kb);
-    // one pipeline step: issue vertex n+2's row loads (s2), vertex n+1's label
-    // gathers (s1), fold vertex n (s0)
-    auto step = [&](int n, Stage &s0, Stage &s1, Stage &s2) {
-        if ((n & (G - 1)) == 0 && n > 0) {
-            // entering group q = n/G: group q+1 goes where group q-1 was, group q+2 is requested
-            if (lane < G) s_ring[wid][(n + G + lane) & (2 * G - 1)] = pend;
-            pend = grec_next();
-            __syncwarp();
-        }
-        load_row(n + 2, s2.ja, s2.jb, s2.wa, s2.wb);
-        gather(n + 1, s1.ja, s1.jb, s1.ka, s1.kb);
-        // ---- fold vertex n ----
+    // pipeline registers: vertex n (fold) / n+1 (gathers in flight) / n+2 (row loads in flight)
+    int32_t j0a, j0b, k0a, k0b, j1a, j1b, k1a, k1b, j2a, j2b;
+    float w0a, w0b, w1a, w1b, w2a, w2b;
+    {
+        load_row(rrec(0), j0a, j0b, w0a, w0b);
+        load_row(rrec(1), j1a, j1b, w1a, w1b);
+        gather(rrec(0).r + (int32_t)a.row_begin, j0a, j0b, k0a, k0b);
+    }
+    uint32_t c_ch = 0, c_che = 0;
+    for (uint32_t n = 0;; ++n) {
         const VRec rc = rrec(n);
+        if (rc.r < 0) break;                               // end record
         const uint32_t dk = r_d(rc);
-        const int64_t ok = r_o(rc);
-        const int64_t vk = rc.r + a.row_begin;
-        Hash h;
-        h.init(dk);
-        TieOrder to;
-        to.init(h);
-        uint32_t bw = 0;
-        int32_t bk = 0;
-        auto offer = [&](float V, int32_t key) {
-            const uint32_t vb = __float_as_uint(V) + 1;
-            if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
-                bw = vb;
-                bk = key;
-            }
-        };
-        auto fold = [&](int32_t key, float w, bool &leader) -> float {
-            const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
-            leader = key != kEmpty && (grp & ((1u << lane) - 1)) == 0;
-            if (W) {
-                const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
-                if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) return (float)__popc(grp) * w;
-                const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-                return maxn > 1 ? group_sum(grp, w, maxn) : w;
-            }
-            return (float)__popc(grp);
-        };
-        const int32_t *pi = a.indices + ok + lane;
-        const float *pw = W ? a.weights + ok + lane : nullptr;
-        auto table_row = [&](auto cap) {
-            constexpr uint32_t P = decltype(cap)::value;
-#pragma unroll
-            for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
+        if ((n & (G - 1)) == 0 && n > 0) {
+            // entering group q = n/G (groups q-1, q in the ring): group q+1
+            // (pend) goes where group q-1 was, group q+2 is requested
+            if (lane < G) s_ring[wid][(n + G + lane) & (RING - 1)] = pend;
+            pend = grec(F.next(ws, lane));
             __syncwarp();
-            auto batch = [&](int32_t key, float w) {
-                bool leader;
-                const float x = fold(key, w, leader);
-                if (leader) offer(kv_add<P>(tab, key, x), key);
-                __syncwarp();
-            };
-            batch(s0.ka, s0.wa);
-            batch(s0.kb, s0.wb);
-            for (uint32_t b = 64; b < dk; b += 32 * U) {
-                // U batches per step: all index loads, then all label gathers in flight
-                int32_t iu[U], qu[U];
-                float xu[U];
-#pragma unroll
-                for (int u = 0; u < U; ++u) {
-                    const bool ok = b + 32 * u + lane < dk;
-                    iu[u] = ok ? ld_stream(pi + b + 32 * u) : -1;
-                    xu[u] = 1.0f;
-                    if (W && ok) xu[u] = ld_stream(pw + b + 32 * u);
-                }
-#pragma unroll
-                for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != (int32_t)vk) ? a.lab_in[iu[u]] : kEmpty;
-#pragma unroll
-                for (int u = 0; u < U; ++u)
-                    if (u == 0 || b + 32 * u < dk) batch(qu[u], xu[u]);
-            }
+        }
+        load_row(rrec(n + 2), j2a, j2b, w2a, w2b);
+        gather(rrec(n + 1).r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
+        // ---- fold vertex n ----
+        const int32_t vk = rc.r + (int32_t)a.row_begin;
+        uint32_t bw = 0;                                   // best (weight bits + 1) this lane led; 0 = none
+        int32_t bk = 0;
+        // unit weights stored (the paper's default weight 1) in the first 64
+        // entries?  Then a group's total is its size (exact); else a
+        // pairwise tree over the group's weights
+        bool eqw = true;
+        if (W) eqw = __all_sync(0xFFFFFFFFu, (k0a == kEmpty || w0a == 1.0f) && (k0b == kEmpty || w0b == 1.0f));
+        auto group_total = [&](unsigned grp, int32_t key, float w, bool eq) -> float {
+            if (!W || eq) return (float)__popc(grp);
+            const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+            return maxn > 1 ? group_sum(grp, w, maxn) : w;
         };
         if (dk <= 32) {
-            bool leader;
-            const float x = fold(s0.ka, s0.wa, leader);
-            if (leader) offer(x, s0.ka);
-        } else if constexpr (SLOTS == kWideSlots) {
-            table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
+            const unsigned grp = __match_any_sync(0xFFFFFFFFu, k0a);
+            const bool leader = k0a != kEmpty && (grp & lanes_below) == 0;
+            const float x = group_total(grp, k0a, w0a, eqw);
+            bw = leader ? __float_as_uint(x) + 1 : 0u;
+            bk = k0a;
         } else {
-            if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
-            else table_row(std::integral_constant<uint32_t, 511>());
+            auto table_row = [&](auto cap) {
+                constexpr uint32_t P = decltype(cap)::value;
+#pragma unroll
+                for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
+                __syncwarp();
+                auto batch = [&](int32_t key, float w, bool eq) {
+                    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+                    const bool leader = key != kEmpty && (grp & lanes_below) == 0;
+                    const float x = group_total(grp, key, w, eq);
+                    const float V = kv_add<P>(tab, key, x, leader);
+                    // running best (total, smallest label) as one 64-bit max
+                    const uint64_t c = ((uint64_t)(__float_as_uint(V) + 1) << 32) | (uint32_t)~key;
+                    const uint64_t b = ((uint64_t)bw << 32) | (uint32_t)~bk;
+                    if (leader && c > b) {
+                        bw = (uint32_t)(c >> 32);
+                        bk = key;
+                    }
+                    __syncwarp();
+                };
+                batch(k0a, w0a, eqw);
+                batch(k0b, w0b, eqw);
+                const int32_t *pi = a.indices + r_o(rc) + lane;
+                const float *pw = W ? a.weights + r_o(rc) + lane : nullptr;
+                for (uint32_t b = 64; b < dk; b += 32 * U) {
+                    // U batches per step: all index loads, then all label gathers in flight
+                    int32_t iu[U], qu[U];
+                    float xu[U];
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        const bool ok = b + 32 * u + lane < dk;
+                        iu[u] = ok ? ld_stream(pi + b + 32 * u) : -1;
+                        xu[u] = 1.0f;
+                        if (W && ok) xu[u] = ld_stream(pw + b + 32 * u);
+                    }
+#pragma unroll
+                    for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != vk) ? lab_in[iu[u]] : kEmpty;
+                    bool eq = true;
+                    if (W) {
+                        bool e = true;
+#pragma unroll
+                        for (int u = 0; u < U; ++u) e = e && (qu[u] == kEmpty || xu[u] == 1.0f);
+                        eq = __all_sync(0xFFFFFFFFu, e);
+                    }
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (u == 0 || b + 32 * u < dk) batch(qu[u], xu[u], eq);
+                }
+            };
+            if constexpr (SLOTS == kWideSlots) {
+                table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
+            } else {
+                if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
+                else table_row(std::integral_constant<uint32_t, 511>());
+            }
         }
+        // hashtableMaxKey: the largest total, ties to the smallest label (R6)
         const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
-        int32_t cs = kEmpty;
-        if (W1) {
-            const uint32_t rr = bw == W1 ? 0xFFFFFFFFu - to.rank(bk) : 0u;
-            cs = to.unrank(0xFFFFFFFFu - __reduce_max_sync(0xFFFFFFFFu, rr));
-        }
+        const int32_t cs = W1 ? (int32_t)__reduce_min_sync(0xFFFFFFFFu, bw == W1 ? (uint32_t)bk : 0xFFFFFFFFu) : kEmpty;
         if (accept_move(cs, rc.ci, a.pickless)) {
             c_ch += 1;
             c_che += dk;
             if (lane == 0) a.lab_out[vk] = cs;
             if (!SYNC) {
                 // vertex n+1's labels were gathered before this write: patch them
-                if (s1.ja == (int32_t)vk) s1.ka = cs;
-                if (s1.jb == (int32_t)vk) s1.kb = cs;
+                if (j1a == vk) k1a = cs;
+                if (j1b == vk) k1b = cs;
             }
-            if (s0.ja >= 0) a.flag_out[s0.ja] = 1;        // mark neighbours unprocessed
-            if (s0.jb >= 0) a.flag_out[s0.jb] = 1;
-            for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[pi[b - lane]] = 1;
+            if (j0a >= 0) a.flag_out[j0a] = 1;            // mark neighbours unprocessed
+            if (j0b >= 0) a.flag_out[j0b] = 1;
+            if (dk > 64) {
+                const int32_t *pi = a.indices + r_o(rc);
+                for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[pi[b]] = 1;
+            }
         }
-    };
-    // (unrolling by 3 so the stages rotate by renaming overflows the instruction cache: 30% slower)
-    for (int n = 0; r_d(rrec(n)) != 0; ++n) {           // records have degree >= 1; zero record = end
-        step(n, SA, SB, SC);
-        SA = SB;
-        SB = SC;
+        // rotate the pipeline
+        j0a = j1a; j0b = j1b; k0a = k1a; k0b = k1b; w0a = w1a; w0b = w1b;
+        j1a = j2a; j1b = j2b; w1a = w2a; w1b = w2b;
     }
     if (lane == 0 && c_ch) {
-        atomicAdd(&bctr[0], c_ch);
-        atomicAdd(&bctr[1], c_che);
+        atomicAdd(&bctr[0], (unsigned long long)c_ch);
+        atomicAdd(&bctr[1], (unsigned long long)c_che);
     }
     __syncthreads();
     if (threadIdx.x == 0 && bctr[0]) {
@@ -1541,6 +1618,7 @@ struct nulpa_graph {
     bool bins_built = false;
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
     void *wrecs = nullptr;          // warp-bin frontier records (VRec [bin_n[1]])
+    unsigned long long *wranges = nullptr;   // SCHED_STEAL: one {next, end} group range per k_warp warp
     void *brecs = nullptr;          // block-bin frontier records (VRec [2 * bin_n[2]]: warp part | CTA part)
     int64_t bin_n[4] = {0, 0, 0, 0};
     int64_t bin_e[4] = {0, 0, 0, 0};
@@ -1626,6 +1704,8 @@ void free_bins(nulpa_graph *g) {
     if (g->stream) cudaStreamSynchronize(g->stream);
     dfree(g->wrecs);
     g->wrecs = nullptr;
+    dfree(g->wranges);
+    g->wranges = nullptr;
     dfree(g->brecs);
     g->brecs = nullptr;
     for (int b = 0; b < 4; ++b) {
@@ -1692,6 +1772,11 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
     CU(cudaMemcpyAsync(ht, totals, sizeof ht, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaMemcpyAsync(he, edges, sizeof he, cudaMemcpyDeviceToHost, g->stream));
     CU(cudaStreamSynchronize(g->stream));
+    {
+        const size_t nwmax = (size_t)num_sms() * kWarpCtasPerSm * kWarpWarps;
+        CHECK(dalloc(&g->wranges, nwmax));
+        CU(cudaMemsetAsync(g->wranges, 0, nwmax * sizeof(unsigned long long), g->stream));   // all ranges empty
+    }
     BinLists L;
     for (int b = 0; b < 4; ++b) {
         g->bin_n[b] = ht[b];
@@ -1777,8 +1862,8 @@ int validate_params(const nulpa_params &p) {
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST) return fail(NULPA_EINVAL, "tie_rule must be NULPA_TIE_SMALLEST (0): ties go to the smallest label (R6)");
     if (p.bin_order < 0 || p.bin_order > 3) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2 or 3");
-    if (p.first_sweep_block < 1 || p.first_sweep_block > 1024 || p.sweep_block < 1 || p.sweep_block > 1024)
-        return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [1, 1024]");
+    if (p.first_sweep_block < 0 || p.first_sweep_block > 1024 || p.sweep_block < 0 || p.sweep_block > 1024)
+        return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [0, 1024]");
     if (p.wide_degree < 1 || p.wide_degree > 1024)   // distinct labels <= D <= 1023 = p1 (R5 always finds a slot)
         return fail(NULPA_EINVAL, "wide_degree must be in [1, 1024] (wide warp tables hold 1023 slots)");
     if (p.giant_degree < p.block_degree || p.giant_degree > 4096)
@@ -1816,8 +1901,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     a.weights = g->weights;
     a.row_begin = g->row_begin;
     a.pickless = pickless;
-    a.sched_block = g->sweeps_since_reset == 0 ? p.first_sweep_block : p.sweep_block;
-    a.split = NULPA_FIRST_SPLIT && g->sweeps_since_reset == 0 && p.first_sweep_block > 1;
+    const int sched_block = g->sweeps_since_reset == 0 ? p.first_sweep_block : p.sweep_block;
     a.ctr = ctr;
     if (SYNC) {
         CU(cudaMemcpyAsync(g->labels_prev, g->labels, g->n_global * sizeof(int32_t), cudaMemcpyDeviceToDevice, g->stream));
@@ -1879,8 +1963,8 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[2], n, 2, rw, ctr + kCtrRecsW,
                                                                           split, rb, ctr + kCtrRecsB);
             if (split > (uint32_t)p.block_degree) {
-                k_warp<SYNC, W, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2,
-                                                                                               ctr + kCtrSchedB);
+                const WarpSched ws{SCHED_GUIDED, NULPA_WIDE_K, ctr + kCtrSchedB, nullptr};
+                k_warp<SYNC, W, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
                 g->stats.launches[2] += 1;
             }
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
@@ -1901,16 +1985,19 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[1], n, 1, recs, ctr + kCtrRecs,
                                                                           0xFFFFFFFFu, nullptr, nullptr);
             if (mid_fork) CU(cudaEventRecord(g->ev_mid, cs));
-            // first-sweep runs of up to K groups need >= K*32 rows per warp: on a
-            // small bin (a row shard of a multi-GPU run) launch fewer CTAs per SM
-            // so each warp still walks long runs (modularity)
-            int ctas = kWarpCtasPerSm;
-            if (a.sched_block > 1 && g->sweeps_since_reset == 0) {
-                const int64_t per = (int64_t)a.sched_block * 32 * kWarpWarps * sms;
-                ctas = (int)std::max<int64_t>(1, std::min<int64_t>(kWarpCtasPerSm, n / per));
+            WarpSched ws{sched_block == 0 ? SCHED_STEAL : sched_block == 1 ? SCHED_STRIDED : SCHED_GUIDED,
+                         sched_block, ctr + kCtrSchedW, g->wranges};
+            int grid = sms * kWarpCtasPerSm;
+            if (ws.mode == SCHED_STEAL) {
+                // each warp walks one run of bin / warps rows; on a small bin
+                // (a test graph, a row shard of a multi-GPU run) launch only
+                // enough warps for runs of >= kMinFirstRun rows (modularity:
+                // labels propagate along ID order within a run)
+                ws.K = (int)(kMinFirstRun / 32);
+                const int64_t warps = std::max<int64_t>(1, n / kMinFirstRun);
+                grid = (int)std::min<int64_t>(grid, (warps + kWarpWarps - 1) / kWarpWarps);
             }
-            k_warp<SYNC, W, kWarpSlots><<<sms * ctas, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1,
-                                                                                          ctr + kCtrSchedW);
+            k_warp<SYNC, W, kWarpSlots><<<grid, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1, ws);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
         }
@@ -2102,7 +2189,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->tie_rule = NULPA_TIE_SMALLEST;
     p->bin_order = 3;
     p->wide_degree = 512;
-    p->first_sweep_block = 192;
+    p->first_sweep_block = 0;
     p->sweep_block = 4;
 }
 

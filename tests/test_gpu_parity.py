@@ -351,16 +351,17 @@ def test_invalid_params_raise():
     with pytest.raises(nl.NulpaError):
         gg.run(wide_degree=1025)
     with pytest.raises(nl.NulpaError):
-        gg.run(first_sweep_block=0)
+        gg.run(first_sweep_block=-1)
     with pytest.raises(nl.NulpaError):
         gg.run(sweep_block=2000)
     with pytest.raises(nl.NulpaError):
         gg.run(tie_rule=1)
 
 
-# warp-bin schedules: (first_sweep_block, sweep_block); 3 and 5 leave ragged
-# last rounds on every test graph
-SCHEDULES = [(1, 1), (3, 5), (128, 1), (1024, 1024)]
+# warp-bin schedules: (first_sweep_block, sweep_block); 0 = contiguous ranges
+# with work stealing (the first-sweep default), 1 = strided, > 1 = guided
+# chunks; 3 and 5 leave ragged last rounds on every test graph
+SCHEDULES = [(0, 4), (0, 0), (1, 1), (3, 5), (128, 1), (1024, 1024)]
 
 
 @pytest.mark.parametrize("gname", ["sbm", "web", "rmat", "kmer"])
