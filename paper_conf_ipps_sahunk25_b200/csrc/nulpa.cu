@@ -778,7 +778,9 @@ struct GroupFetcher {
     }
 };
 
-template <bool SYNC, bool W, int SLOTS>
+// O32: every CSR offset + 64 fits 32 bits (M < 2^32 - 64): row addresses
+// are one 32-bit add + IMAD.WIDE instead of 48-bit arithmetic.
+template <bool SYNC, bool W, int SLOTS, bool O32>
 __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ctas)
     k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin,
            WarpSched ws) {
@@ -788,7 +790,9 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     constexpr uint32_t RING = 2 * G;
     static_assert(G >= 1 && G <= 32 && (G & (G - 1)) == 0, "group size: power of two <= 32");
     __shared__ __align__(16) uint64_t s_tab[NWARP][SLOTS];
-    __shared__ __align__(16) VRec s_ring[NWARP][RING];   // two groups; record m sits at m mod 2G
+    // two groups; record m sits at m mod 2G, and records 0, 1 again at 2G,
+    // 2G+1 (so records n+1, n+2 are at fixed offsets from record n)
+    __shared__ __align__(16) VRec s_ring[NWARP][RING + 2];
     __shared__ unsigned long long bctr[2];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const uint32_t tab = (uint32_t)__cvta_generic_to_shared(&s_tab[wid][0]);
@@ -821,36 +825,44 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         const uint32_t i = g * G + lane;
         return i < nrec ? recs[i] : VRec{0, 0, 0, 0};
     };
-    auto rrec = [&](uint32_t m) -> VRec {
+    auto rrec_at = [&](uint32_t addr) -> VRec {
         VRec r;
         asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
                      : "=r"(r.o_lo), "=r"(r.o_hi_deg), "=r"(r.r), "=r"(r.ci)
-                     : "r"(ring + 16u * (m & (RING - 1))) : "memory");
+                     : "r"(addr) : "memory");
         return r;
     };
-    auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
+    // row offset (48 bit; 32 bit under O32) and degree of a record
+    auto r_o = [](const VRec &r) -> uint64_t {
+        return O32 ? (uint64_t)r.o_lo : ((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo;
+    };
     auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
+    // group -> ring slots [base, base + G) (+ the copy of records 0, 1)
+    auto ring_put = [&](uint32_t base, const VRec &r) {
+        if (lane < G) s_ring[wid][base + lane] = r;
+        if (base == 0 && lane < 2) s_ring[wid][RING + lane] = r;
+    };
     {
         const VRec r0 = grec(F.next(ws, lane));
         const VRec r1 = grec(F.next(ws, lane));
-        if (lane < G) {
-            s_ring[wid][lane] = r0;
-            s_ring[wid][G + lane] = r1;
-        }
+        ring_put(0, r0);
+        ring_put(G, r1);
     }
     VRec pend = grec(F.next(ws, lane));
     __syncwarp();
     const int32_t *__restrict__ lab_in = a.lab_in;
     // row loads: entries lane and lane+32 of the row of record m
+    // entry e of the CSR arrays (e = row offset + position)
+    auto at = [&](uint64_t o, uint32_t k) -> uint64_t { return O32 ? (uint64_t)((uint32_t)o + k) : o + k; };
     auto load_row = [&](const VRec &r, int32_t &ja, int32_t &jb, float &wa, float &wb) {
         const uint32_t d = r_d(r);
-        const int64_t o = r_o(r);
-        const int32_t *pi = a.indices + o + lane;
+        const uint64_t e = at(r_o(r), (uint32_t)lane);
+        const int32_t *pi = a.indices + e;
         ja = (uint32_t)lane < d ? ld_stream(pi) : -1;
         jb = (uint32_t)lane + 32 < d ? ld_stream(pi + 32) : -1;
         wa = wb = 1.0f;
         if (W) {
-            const float *pw = a.weights + o + lane;
+            const float *pw = a.weights + e;
             if ((uint32_t)lane < d) wa = ld_stream(pw);
             if ((uint32_t)lane + 32 < d) wb = ld_stream(pw + 32);
         }
@@ -864,24 +876,27 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     int32_t j0a, j0b, k0a, k0b, j1a, j1b, k1a, k1b, j2a, j2b;
     float w0a, w0b, w1a, w1b, w2a, w2b;
     {
-        load_row(rrec(0), j0a, j0b, w0a, w0b);
-        load_row(rrec(1), j1a, j1b, w1a, w1b);
-        gather(rrec(0).r + (int32_t)a.row_begin, j0a, j0b, k0a, k0b);
+        load_row(rrec_at(ring), j0a, j0b, w0a, w0b);
+        load_row(rrec_at(ring + 16), j1a, j1b, w1a, w1b);
+        gather(rrec_at(ring).r + (int32_t)a.row_begin, j0a, j0b, k0a, k0b);
     }
     uint32_t c_ch = 0, c_che = 0;
-    for (uint32_t n = 0;; ++n) {
-        const VRec rc = rrec(n);
-        if (rc.r < 0) break;                               // end record
+    for (uint32_t q = 0;; ++q) {                           // record groups
+      if (q > 0) {
+          // entering group q (groups q-1, q in the ring): group q+1 (pend)
+          // goes where group q-1 was, group q+2 is requested
+          ring_put(((q + 1) & 1) * G, pend);
+          pend = grec(F.next(ws, lane));
+          __syncwarp();
+      }
+      const uint32_t ring_q = ring + 16u * ((q & 1) * G);
+      for (uint32_t p = 0; p < (uint32_t)G; ++p) {          // vertex n = q*G + p
+        const uint32_t rn = ring_q + 16u * p;
+        const VRec rc = rrec_at(rn);
+        if (rc.r < 0) goto done;                           // end record
         const uint32_t dk = r_d(rc);
-        if ((n & (G - 1)) == 0 && n > 0) {
-            // entering group q = n/G (groups q-1, q in the ring): group q+1
-            // (pend) goes where group q-1 was, group q+2 is requested
-            if (lane < G) s_ring[wid][(n + G + lane) & (RING - 1)] = pend;
-            pend = grec(F.next(ws, lane));
-            __syncwarp();
-        }
-        load_row(rrec(n + 2), j2a, j2b, w2a, w2b);
-        gather(rrec(n + 1).r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
+        load_row(rrec_at(rn + 32), j2a, j2b, w2a, w2b);
+        gather(rrec_at(rn + 16).r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
         // ---- fold vertex n ----
         const int32_t vk = rc.r + (int32_t)a.row_begin;
         uint32_t bw = 0;                                   // best (weight bits + 1) this lane led; 0 = none
@@ -924,8 +939,9 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
                 };
                 batch(k0a, w0a, eqw);
                 batch(k0b, w0b, eqw);
-                const int32_t *pi = a.indices + r_o(rc) + lane;
-                const float *pw = W ? a.weights + r_o(rc) + lane : nullptr;
+                const uint64_t el = at(r_o(rc), (uint32_t)lane);
+                const int32_t *pi = a.indices + el;
+                const float *pw = W ? a.weights + el : nullptr;
                 for (uint32_t b = 64; b < dk; b += 32 * U) {
                     // U batches per step: all index loads, then all label gathers in flight
                     int32_t iu[U], qu[U];
@@ -972,15 +988,14 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
             }
             if (j0a >= 0) a.flag_out[j0a] = 1;            // mark neighbours unprocessed
             if (j0b >= 0) a.flag_out[j0b] = 1;
-            if (dk > 64) {
-                const int32_t *pi = a.indices + r_o(rc);
-                for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[pi[b]] = 1;
-            }
+            for (uint32_t b = 64 + lane; b < dk; b += 32) a.flag_out[a.indices[at(r_o(rc), b)]] = 1;
         }
         // rotate the pipeline
         j0a = j1a; j0b = j1b; k0a = k1a; k0b = k1b; w0a = w1a; w0b = w1b;
         j1a = j2a; j1b = j2b; w1a = w2a; w1b = w2b;
+      }
     }
+done:
     if (lane == 0 && c_ch) {
         atomicAdd(&bctr[0], (unsigned long long)c_ch);
         atomicAdd(&bctr[1], (unsigned long long)c_che);
@@ -1917,6 +1932,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     a.lab_out = g->labels;
     a.flag_out = g->flags;
     const int sms = num_sms();
+    const bool o32 = g->M + 64 < (INT64_C(1) << 32);  // 32-bit row addressing in k_warp
     cudaStream_t cs = g->stream;                  // stream of the bin being launched
     auto rec = [&](int b, int which) -> int {
         if (timing) CU(cudaEventRecord(g->ev[(slot * 4 + b) * 2 + which], cs));
@@ -1964,7 +1980,10 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                                                                           split, rb, ctr + kCtrRecsB);
             if (split > (uint32_t)p.block_degree) {
                 const WarpSched ws{SCHED_GUIDED, NULPA_WIDE_K, ctr + kCtrSchedB, nullptr};
-                k_warp<SYNC, W, kWideSlots><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
+                if (o32)
+                    k_warp<SYNC, W, kWideSlots, true><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
+                else
+                    k_warp<SYNC, W, kWideSlots, false><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
                 g->stats.launches[2] += 1;
             }
             const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
@@ -1997,7 +2016,10 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                 const int64_t warps = std::max<int64_t>(1, n / kMinFirstRun);
                 grid = (int)std::min<int64_t>(grid, (warps + kWarpWarps - 1) / kWarpWarps);
             }
-            k_warp<SYNC, W, kWarpSlots><<<grid, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1, ws);
+            if (o32)
+                k_warp<SYNC, W, kWarpSlots, true><<<grid, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1, ws);
+            else
+                k_warp<SYNC, W, kWarpSlots, false><<<grid, kWarpWarps * 32, 0, cs>>>(a, recs, ctr + kCtrRecs, 1, ws);
             CU(cudaGetLastError());
             g->stats.launches[1] += 2;
         }
