@@ -235,40 +235,13 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
     return x;
 }
 
-// Shared-memory accessors with 32-bit shared-window addresses (the k_warp
-// tables); "memory" clobbers keep table reads/writes in program order.
-__device__ __forceinline__ uint64_t lds_u64(uint32_t addr) {
-    uint64_t v;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(addr) : "memory");
-    return v;
-}
-__device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
-    asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
-}
 // k_warp tables store the tag k + 1 for label k (labels are >= 0 and < 2^31 - 1),
 // so an empty slot (tag 0, value 0.0f) is all-zero and hashtableClear is a
 // 16-byte store of the zero register (no per-vertex register set-up).
-#ifndef NULPA_ZERO_EMPTY
-#define NULPA_ZERO_EMPTY 1
-#endif
-#if NULPA_ZERO_EMPTY
 constexpr uint32_t kTagEmpty = 0u;
 __device__ __forceinline__ uint32_t kv_tag(int32_t k) { return (uint32_t)k + 1u; }
 __device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
     asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(addr), "r"(0u) : "memory");
-}
-#else
-constexpr uint32_t kTagEmpty = 0xFFFFFFFFu;
-__device__ __forceinline__ uint32_t kv_tag(int32_t k) { return (uint32_t)k; }
-__device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
-    // two empty slots: key = phi (0xFFFFFFFF), value = 0.0f
-    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %1, %2};" ::"r"(addr), "r"(0xFFFFFFFFu), "r"(0u) : "memory");
-}
-#endif
-__device__ __forceinline__ uint32_t cas_u32(uint32_t addr, uint32_t cmp, uint32_t val) {
-    uint32_t old;
-    asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "r"(addr), "r"(cmp), "r"(val) : "memory");
-    return old;
 }
 
 // (weight, tie rank) packed so that an unsigned max gives the largest weight
@@ -778,6 +751,99 @@ struct GroupFetcher {
     }
 };
 
+// The fold of one vertex by one warp (lines 337-343 of Algorithm 1): the
+// first 64 row entries arrive as labels k0a / k0b (entries lane, lane + 32;
+// kEmpty = absent or the vertex itself) with weights w0a / w0b, later entries
+// are loaded here.  Returns hashtableMaxKey (kEmpty if no neighbour).
+template <bool W, int SLOTS, bool O32>
+__device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, int lane, unsigned lanes_below,
+                                             uint64_t row_o, uint32_t dk, int32_t vk, int32_t k0a, int32_t k0b,
+                                             float w0a, float w0b) {
+    constexpr int U = WarpCfg<SLOTS>::unroll;
+    (void)U;
+    const int32_t *__restrict__ lab_in = a.lab_in;
+    auto at = [&](uint64_t o, uint32_t k) -> uint64_t { return O32 ? (uint64_t)((uint32_t)o + k) : o + k; };
+    uint32_t bw = 0;                                       // best (weight bits + 1) this lane led; 0 = none
+    int32_t bk = 0;
+    // unit weights stored (the paper's default weight 1) in the first 64
+    // entries?  Then a group's total is its size (exact); else a
+    // pairwise tree over the group's weights
+    bool eqw = true;
+    if (W) eqw = __all_sync(0xFFFFFFFFu, (k0a == kEmpty || w0a == 1.0f) && (k0b == kEmpty || w0b == 1.0f));
+    auto group_total = [&](unsigned grp, int32_t key, float w, bool eq) -> float {
+        if (!W || eq) return (float)__popc(grp);
+        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
+        return maxn > 1 ? group_sum(grp, w, maxn) : w;
+    };
+    if (dk <= 32) {
+        const unsigned grp = __match_any_sync(0xFFFFFFFFu, k0a);
+        const bool leader = k0a != kEmpty && (grp & lanes_below) == 0;
+        const float x = group_total(grp, k0a, w0a, eqw);
+        bw = leader ? __float_as_uint(x) + 1 : 0u;
+        bk = k0a;
+    } else {
+        auto table_row = [&](auto cap) {
+            constexpr uint32_t P = decltype(cap)::value;
+#pragma unroll
+            for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
+            __syncwarp();
+            auto batch = [&](int32_t key, float w, bool eq) {
+                const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
+                const bool leader = key != kEmpty && (grp & lanes_below) == 0;
+                const float x = group_total(grp, key, w, eq);
+                const float V = kv_add<P>(tab, key, x, leader);
+                // running best (total, smallest label) as one 64-bit max
+                const uint64_t c = ((uint64_t)(__float_as_uint(V) + 1) << 32) | (uint32_t)~key;
+                const uint64_t b = ((uint64_t)bw << 32) | (uint32_t)~bk;
+                if (leader && c > b) {
+                    bw = (uint32_t)(c >> 32);
+                    bk = key;
+                }
+                __syncwarp();
+            };
+            batch(k0a, w0a, eqw);
+            batch(k0b, w0b, eqw);
+            const uint64_t el = at(row_o, (uint32_t)lane);
+            const int32_t *pi = a.indices + el;
+            const float *pw = W ? a.weights + el : nullptr;
+            for (uint32_t b = 64; b < dk; b += 32 * U) {
+                // U batches per step: all index loads, then all label gathers in flight
+                int32_t iu[U], qu[U];
+                float xu[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const bool ok = b + 32 * u + lane < dk;
+                    iu[u] = ok ? ld_stream(pi + b + 32 * u) : -1;
+                    xu[u] = 1.0f;
+                    if (W && ok) xu[u] = ld_stream(pw + b + 32 * u);
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != vk) ? lab_in[iu[u]] : kEmpty;
+                bool eq = true;
+                if (W) {
+                    bool e = true;
+#pragma unroll
+                    for (int u = 0; u < U; ++u) e = e && (qu[u] == kEmpty || xu[u] == 1.0f);
+                    eq = __all_sync(0xFFFFFFFFu, e);
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (u == 0 || b + 32 * u < dk) batch(qu[u], xu[u], eq);
+            }
+        };
+        if constexpr (SLOTS == kWideSlots) {
+            table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
+        } else {
+            if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
+            else table_row(std::integral_constant<uint32_t, 511>());
+        }
+    }
+    // hashtableMaxKey: the largest total, ties to the smallest label (R6)
+    const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
+    const int32_t cs = W1 ? (int32_t)__reduce_min_sync(0xFFFFFFFFu, bw == W1 ? (uint32_t)bk : 0xFFFFFFFFu) : kEmpty;
+    return cs;
+}
+
 // O32: every CSR offset + 64 fits 32 bits (M < 2^32 - 64): row addresses
 // are one 32-bit add + IMAD.WIDE instead of 48-bit arithmetic.
 template <bool SYNC, bool W, int SLOTS, bool O32>
@@ -899,84 +965,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         gather(rrec_at(rn + 16).r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
         // ---- fold vertex n ----
         const int32_t vk = rc.r + (int32_t)a.row_begin;
-        uint32_t bw = 0;                                   // best (weight bits + 1) this lane led; 0 = none
-        int32_t bk = 0;
-        // unit weights stored (the paper's default weight 1) in the first 64
-        // entries?  Then a group's total is its size (exact); else a
-        // pairwise tree over the group's weights
-        bool eqw = true;
-        if (W) eqw = __all_sync(0xFFFFFFFFu, (k0a == kEmpty || w0a == 1.0f) && (k0b == kEmpty || w0b == 1.0f));
-        auto group_total = [&](unsigned grp, int32_t key, float w, bool eq) -> float {
-            if (!W || eq) return (float)__popc(grp);
-            const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-            return maxn > 1 ? group_sum(grp, w, maxn) : w;
-        };
-        if (dk <= 32) {
-            const unsigned grp = __match_any_sync(0xFFFFFFFFu, k0a);
-            const bool leader = k0a != kEmpty && (grp & lanes_below) == 0;
-            const float x = group_total(grp, k0a, w0a, eqw);
-            bw = leader ? __float_as_uint(x) + 1 : 0u;
-            bk = k0a;
-        } else {
-            auto table_row = [&](auto cap) {
-                constexpr uint32_t P = decltype(cap)::value;
-#pragma unroll
-                for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
-                __syncwarp();
-                auto batch = [&](int32_t key, float w, bool eq) {
-                    const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
-                    const bool leader = key != kEmpty && (grp & lanes_below) == 0;
-                    const float x = group_total(grp, key, w, eq);
-                    const float V = kv_add<P>(tab, key, x, leader);
-                    // running best (total, smallest label) as one 64-bit max
-                    const uint64_t c = ((uint64_t)(__float_as_uint(V) + 1) << 32) | (uint32_t)~key;
-                    const uint64_t b = ((uint64_t)bw << 32) | (uint32_t)~bk;
-                    if (leader && c > b) {
-                        bw = (uint32_t)(c >> 32);
-                        bk = key;
-                    }
-                    __syncwarp();
-                };
-                batch(k0a, w0a, eqw);
-                batch(k0b, w0b, eqw);
-                const uint64_t el = at(r_o(rc), (uint32_t)lane);
-                const int32_t *pi = a.indices + el;
-                const float *pw = W ? a.weights + el : nullptr;
-                for (uint32_t b = 64; b < dk; b += 32 * U) {
-                    // U batches per step: all index loads, then all label gathers in flight
-                    int32_t iu[U], qu[U];
-                    float xu[U];
-#pragma unroll
-                    for (int u = 0; u < U; ++u) {
-                        const bool ok = b + 32 * u + lane < dk;
-                        iu[u] = ok ? ld_stream(pi + b + 32 * u) : -1;
-                        xu[u] = 1.0f;
-                        if (W && ok) xu[u] = ld_stream(pw + b + 32 * u);
-                    }
-#pragma unroll
-                    for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != vk) ? lab_in[iu[u]] : kEmpty;
-                    bool eq = true;
-                    if (W) {
-                        bool e = true;
-#pragma unroll
-                        for (int u = 0; u < U; ++u) e = e && (qu[u] == kEmpty || xu[u] == 1.0f);
-                        eq = __all_sync(0xFFFFFFFFu, e);
-                    }
-#pragma unroll
-                    for (int u = 0; u < U; ++u)
-                        if (u == 0 || b + 32 * u < dk) batch(qu[u], xu[u], eq);
-                }
-            };
-            if constexpr (SLOTS == kWideSlots) {
-                table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
-            } else {
-                if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
-                else table_row(std::integral_constant<uint32_t, 511>());
-            }
-        }
-        // hashtableMaxKey: the largest total, ties to the smallest label (R6)
-        const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
-        const int32_t cs = W1 ? (int32_t)__reduce_min_sync(0xFFFFFFFFu, bw == W1 ? (uint32_t)bk : 0xFFFFFFFFu) : kEmpty;
+        const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, k0a, k0b, w0a, w0b);
         if (accept_move(cs, rc.ci, a.pickless)) {
             c_ch += 1;
             c_che += dk;
