@@ -113,6 +113,12 @@ typedef struct nulpa_stats {
     int64_t bin_vertices[4];           /* vertices in each degree bin                  */
     int64_t bin_edges[4];              /* CSR entries of the vertices in each bin      */
     double run_ms;                     /* wall time of nulpa_run on the stream (events) */
+    /* per iteration l < 64 and bin b (the totals above split by iteration):  */
+    double iter_kernel_ms[64][4];      /* bin b's event span in iteration l (timing=1)  */
+    int64_t iter_processed[64][4];
+    int64_t iter_edges[64][4];
+    int64_t iter_changed[64][4];
+    int64_t iter_changed_edges[64][4];
 } nulpa_stats;
 
 void nulpa_default_params(nulpa_params *p);

@@ -72,6 +72,11 @@ class Stats(ctypes.Structure):
         ("bin_vertices", ctypes.c_int64 * 4),
         ("bin_edges", ctypes.c_int64 * 4),
         ("run_ms", ctypes.c_double),
+        ("iter_kernel_ms", (ctypes.c_double * 4) * 64),
+        ("iter_processed", (ctypes.c_int64 * 4) * 64),
+        ("iter_edges", (ctypes.c_int64 * 4) * 64),
+        ("iter_changed", (ctypes.c_int64 * 4) * 64),
+        ("iter_changed_edges", (ctypes.c_int64 * 4) * 64),
     ]
 
     def to_dict(self) -> dict:
@@ -83,6 +88,9 @@ class Stats(ctypes.Structure):
             kernel_ms=list(self.kernel_ms),
             launches=list(self.launches), other_launches=self.other_launches,
             bin_vertices=list(self.bin_vertices), bin_edges=list(self.bin_edges), run_ms=self.run_ms,
+            per_iteration=[dict(kernel_ms=list(self.iter_kernel_ms[l]), processed=list(self.iter_processed[l]),
+                                edges=list(self.iter_edges[l]), changed=list(self.iter_changed[l]),
+                                changed_edges=list(self.iter_changed_edges[l])) for l in range(min(it, 64))],
         )
 
 

@@ -299,33 +299,6 @@ struct SweepArgs {
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 
-// Warp-aggregated (ballot / redux) then CTA-aggregated changed-vertex,
-// processed-vertex and edge counters: one set of global atomics per CTA.
-// bctr: 4 shared counters zeroed before the first __syncthreads.
-__device__ __forceinline__ void block_count(unsigned long long *ctr, unsigned long long *bctr, int bin, bool act,
-                                            bool changed, uint32_t edges) {
-    unsigned m_act = __ballot_sync(0xFFFFFFFFu, act);
-    unsigned m_ch = __ballot_sync(0xFFFFFFFFu, changed);
-    uint32_t e = __reduce_add_sync(0xFFFFFFFFu, edges);
-    uint32_t ec = __reduce_add_sync(0xFFFFFFFFu, changed ? edges : 0u);
-    if ((threadIdx.x & 31) == 0 && m_act) {
-        atomicAdd(&bctr[0], (unsigned long long)__popc(m_act));
-        atomicAdd(&bctr[1], (unsigned long long)e);
-        atomicAdd(&bctr[2], (unsigned long long)__popc(m_ch));
-        atomicAdd(&bctr[3], (unsigned long long)ec);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0 && bctr[0]) {
-        atomicAdd(&ctr[1 + bin], bctr[0]);
-        atomicAdd(&ctr[5 + bin], bctr[1]);
-        if (bctr[2]) {
-            atomicAdd(&ctr[0], bctr[2]);
-            atomicAdd(&ctr[9 + bin], bctr[2]);
-            atomicAdd(&ctr[13 + bin], bctr[3]);
-        }
-    }
-}
-
 // ---------------------------------------------------------------------------
 // thread-per-vertex kernel (degree < switch_degree <= 33), PAPER.md:241-243:
 // "only a single thread operates on the hashtable.  This eliminates the need
@@ -336,63 +309,109 @@ __device__ __forceinline__ void block_count(unsigned long long *ctr, unsigned lo
 // ---------------------------------------------------------------------------
 template <bool SYNC, bool W, int MAXD>
 __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const int32_t *__restrict__ list,
-                                                           int64_t n) {
+                                                           int64_t n, bool consec4) {
+    // Grid-stride over the bin list, 4 consecutive entries per thread and
+    // step: one 16-byte list load and four independent flag loads, then the
+    // unprocessed ones are folded.  Late sweeps of a road network are a scan
+    // of mostly pruned vertices; one entry per thread and step made every
+    // step two dependent round trips (list -> flag) for one entry.
     __shared__ unsigned long long bctr[4];
     if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
     __syncthreads();
-    int64_t t = (int64_t)blockIdx.x * kThreadThreads + threadIdx.x;
-    bool act = false, changed = false;
-    uint32_t deg = 0;
-    if (t < n) {
-        int32_t r = list[t];
-        int64_t v = r + a.row_begin;
-        if (a.flag_in[v]) {
-            act = true;
-            if (!SYNC) a.flag_in[v] = 0;                 // mark i as processed
-            int64_t o = a.offsets[r];
-            deg = (uint32_t)(a.offsets[r + 1] - o);
-            int32_t lab[MAXD];
-            float w[MAXD];
+    uint32_t n_act = 0, n_ch = 0;
+    unsigned long long e_act = 0, e_ch = 0;
+    auto process = [&](int32_t r) {
+        const int64_t v = r + a.row_begin;
+        const int64_t o = a.offsets[r];
+        const uint32_t deg = (uint32_t)(a.offsets[r + 1] - o);
+        int32_t lab[MAXD];
+        float w[MAXD];
 #pragma unroll
-            for (int k = 0; k < MAXD; ++k) {
-                lab[k] = kEmpty;
-                w[k] = 0.0f;
-                if (k < (int)deg) {
-                    int32_t j = a.indices[o + k];
-                    if (j != (int32_t)v) {                // "if j = i continue"
-                        lab[k] = a.lab_in[j];
-                        w[k] = W ? a.weights[o + k] : 1.0f;
-                    }
+        for (int k = 0; k < MAXD; ++k) {
+            lab[k] = kEmpty;
+            w[k] = 0.0f;
+            if (k < (int)deg) {
+                const int32_t j = a.indices[o + k];
+                if (j != (int32_t)v) {                      // "if j = i continue"
+                    lab[k] = a.lab_in[j];
+                    w[k] = W ? a.weights[o + k] : 1.0f;
                 }
-            }
-            Hash h;
-            h.init(deg);
-            TieOrder to;
-            to.init(h);
-            uint64_t best = 0;
-#pragma unroll
-            for (int k = 0; k < MAXD; ++k) {
-                if (k >= (int)deg) break;
-                if (lab[k] == kEmpty) continue;
-                float s = 0.0f;
-#pragma unroll
-                for (int m = 0; m < MAXD; ++m) {
-                    if (m >= (int)deg) break;
-                    s = __fadd_rn(s, lab[m] == lab[k] ? w[m] : 0.0f);
-                }
-                uint64_t c = pack_cand(s, lab[k], to);
-                best = c > best ? c : best;
-            }
-            int32_t ci = a.lab_in[v];
-            int32_t cs = best ? cand_label(best, to) : kEmpty;
-            if (accept_move(cs, ci, a.pickless)) {
-                a.lab_out[v] = cs;
-                changed = true;
-                for (uint32_t k = 0; k < deg; ++k) a.flag_out[a.indices[o + k]] = 1;
             }
         }
+        TieOrder to;
+        uint64_t best = 0;
+#pragma unroll
+        for (int k = 0; k < MAXD; ++k) {
+            if (k >= (int)deg) break;
+            if (lab[k] == kEmpty) continue;
+            float s = 0.0f;
+#pragma unroll
+            for (int m = 0; m < MAXD; ++m) {
+                if (m >= (int)deg) break;
+                s = __fadd_rn(s, lab[m] == lab[k] ? w[m] : 0.0f);
+            }
+            const uint64_t c = pack_cand(s, lab[k], to);
+            best = c > best ? c : best;
+        }
+        const int32_t ci = a.lab_in[v];
+        const int32_t cs = best ? cand_label(best, to) : kEmpty;
+        n_act += 1;
+        e_act += deg;
+        if (accept_move(cs, ci, a.pickless)) {
+            a.lab_out[v] = cs;
+            n_ch += 1;
+            e_ch += deg;
+            for (uint32_t k = 0; k < deg; ++k) a.flag_out[a.indices[o + k]] = 1;
+        }
+    };
+    // step = 4 consecutive entries per thread (bulk bins: ordered sweep,
+    // fewer dependent scan round trips) or 1 (thin bins: all parallelism)
+    const int64_t nq = consec4 ? (n + 3) / 4 : n;
+    for (int64_t q = (int64_t)blockIdx.x * kThreadThreads + threadIdx.x; q < nq; q += (int64_t)gridDim.x * kThreadThreads) {
+        int32_t r[4] = {-1, -1, -1, -1};
+        if (!consec4) {
+            r[0] = list[q];
+        } else if (4 * q + 3 < n) {
+            const int4 v4 = *reinterpret_cast<const int4 *>(list + 4 * q);   // the bin list is 16-byte aligned
+            r[0] = v4.x; r[1] = v4.y; r[2] = v4.z; r[3] = v4.w;
+        } else {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) r[u] = 4 * q + u < n ? list[4 * q + u] : -1;
+        }
+        bool act[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) act[u] = r[u] >= 0 && a.flag_in[r[u] + a.row_begin] != 0;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            if (!act[u]) continue;                          // "if not unprocessed(i) continue"
+            if (!SYNC) a.flag_in[r[u] + a.row_begin] = 0;   // mark i as processed
+            process(r[u]);
+        }
     }
-    block_count(a.ctr, bctr, 0, act, changed, act ? deg : 0);
+    // counters: warp sums, then one set of global atomics per CTA
+    n_act = __reduce_add_sync(0xFFFFFFFFu, n_act);
+    n_ch = __reduce_add_sync(0xFFFFFFFFu, n_ch);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        e_act += __shfl_xor_sync(0xFFFFFFFFu, e_act, o);
+        e_ch += __shfl_xor_sync(0xFFFFFFFFu, e_ch, o);
+    }
+    if ((threadIdx.x & 31) == 0 && n_act) {
+        atomicAdd(&bctr[0], (unsigned long long)n_act);
+        atomicAdd(&bctr[1], e_act);
+        atomicAdd(&bctr[2], (unsigned long long)n_ch);
+        atomicAdd(&bctr[3], e_ch);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && bctr[0]) {
+        atomicAdd(&a.ctr[1], bctr[0]);
+        atomicAdd(&a.ctr[5], bctr[1]);
+        if (bctr[2]) {
+            atomicAdd(&a.ctr[0], bctr[2]);
+            atomicAdd(&a.ctr[9], bctr[2]);
+            atomicAdd(&a.ctr[13], bctr[3]);
+        }
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -668,6 +687,7 @@ enum { SCHED_STRIDED = 0, SCHED_GUIDED = 1, SCHED_STEAL = 2 };
 #define NULPA_MIN_RUN 2048
 #endif
 constexpr int64_t kMinFirstRun = NULPA_MIN_RUN;   // rows per warp in the first sweep, at least (small bins)
+constexpr double kLocalRuns = 0.5;                // ... if >= this share of the sampled CSR entries are near (k_locality)
 struct WarpSched {
     int mode;
     int K;                               // guided chunk size (groups)
@@ -1440,6 +1460,26 @@ __global__ void __launch_bounds__(kBinTile) k_bin_scatter(const int64_t *offsets
     }
 }
 
+// ID locality of the graph (first-sweep schedule, DESIGN.md "Quality
+// notes"): over `ns` sampled rows (every `step`-th), acc[0] += CSR entries,
+// acc[1] += entries whose neighbour ID is within kNear of the row's ID.
+constexpr int64_t kNear = 2048;
+__global__ void k_locality(const int64_t *__restrict__ offsets, const int32_t *__restrict__ indices, int64_t row_begin,
+                           int64_t step, int64_t ns, unsigned long long *acc) {
+    unsigned long long tot = 0, near = 0;
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < ns; s += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = s * step, v = r + row_begin;
+        const int64_t e1 = min(offsets[r + 1], offsets[r] + 64);    // up to 64 entries per sampled row
+        for (int64_t e = offsets[r]; e < e1; ++e) {
+            const int64_t d = (int64_t)indices[e] - v;
+            near += d >= -kNear && d <= kNear;
+            ++tot;
+        }
+    }
+    atomicAdd(&acc[0], tot);
+    atomicAdd(&acc[1], near);
+}
+
 __global__ void k_gather_degrees(const int64_t *offsets, const int32_t *rows, int64_t n, int64_t *out) {
     int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (k < n) {
@@ -1623,6 +1663,7 @@ struct nulpa_graph {
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
     void *wrecs = nullptr;          // warp-bin frontier records (VRec [bin_n[1]])
     unsigned long long *wranges = nullptr;   // SCHED_STEAL: one {next, end} group range per k_warp warp
+    double locality = 0.0;          // share of sampled CSR entries j with |j - i| <= kNear (k_locality)
     void *brecs = nullptr;          // block-bin frontier records (VRec [2 * bin_n[2]]: warp part | CTA part)
     int64_t bin_n[4] = {0, 0, 0, 0};
     int64_t bin_e[4] = {0, 0, 0, 0};
@@ -1845,6 +1886,19 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CU(cudaStreamSynchronize(g->stream));          // before cg / c0 / c1 / toff go out of scope
     }
     CU(cudaStreamSynchronize(g->stream));
+    {
+        // ID locality from <= 65536 sampled rows (reuses `edges` as the accumulator)
+        const int64_t ns = std::min<int64_t>(n, 65536), step = ns ? n / ns : 1;
+        unsigned long long h[2] = {0, 0};
+        if (ns > 0) {
+            CU(cudaMemsetAsync(edges, 0, 2 * sizeof(unsigned long long), g->stream));
+            k_locality<<<grid_for(ns, 256), 256, 0, g->stream>>>(g->offsets, g->indices, g->row_begin, step, ns, edges);
+            CU(cudaGetLastError());
+            CU(cudaMemcpyAsync(h, edges, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+            CU(cudaStreamSynchronize(g->stream));
+        }
+        g->locality = h[0] ? (double)h[1] / (double)h[0] : 0.0;
+    }
     dfree(counts);
     dfree(totals);
     dfree(edges);
@@ -1880,20 +1934,50 @@ int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
     return build_bins(g, p.switch_degree, p.block_degree, p.giant_degree);
 }
 
+// The thread bin in kThreadWaves launches over consecutive slices of the
+// bin list (asynchronous mode, when the thread bin holds at least half of
+// the CSR entries and spans fewer than kThreadWaves grid-stride steps): a
+// vertex of slice w sees the labels slices
+// < w wrote in this sweep, so on graphs whose neighbours have unrelated IDs
+// (k-mer paths, permuted IDs) about half of its neighbours are already
+// updated, as in the sequential ID-order sweep of Algorithm 1 -- one launch
+// over a small bin processes every vertex at once (Jacobi) and lands ~0.02
+// below the sequential sweep's modularity on k-mer graphs.
+#ifndef NULPA_THREAD_WAVES
+#define NULPA_THREAD_WAVES 8
+#endif
+constexpr int kThreadWaves = NULPA_THREAD_WAVES;
 template <bool SYNC, bool W>
 int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const int64_t n = g->bin_n[0];
-    const int grid = grid_for(n, kThreadThreads);
     const int64_t md = g->bin_maxdeg[0];     // register table sized by the bin's largest degree
-    if (md <= 4)
-        k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    else if (md <= 8)
-        k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    else if (md <= 16)
-        k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    else
-        k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, g->bin_list[0], n);
-    CU(cudaGetLastError());
+    // a bin spanning >= kThreadWaves grid-stride steps is already swept in
+    // order (step s of every thread covers entries [4Ts, 4T(s+1))): one launch
+    const int64_t per_step = 4LL * kThreadThreads * num_sms() * 8;
+    // order matters for the sweep's result only where the thread bin is most
+    // of the graph (path-like k-mer / road graphs); elsewhere a thin bin of
+    // low-degree vertices is one launch
+    const bool bulk = 2 * g->bin_e[0] >= g->M;
+    int64_t waves = SYNC || !bulk ? 1 : (kThreadWaves * per_step + n - 1) / std::max<int64_t>(n, 1);
+    waves = std::max<int64_t>(1, std::min<int64_t>({waves, (int64_t)kThreadWaves, n / 1024}));
+    for (int64_t w = 0; w < waves; ++w) {
+        // slice bounds on multiples of 4 entries (k_thread reads the list 16 bytes at a time)
+        const int64_t b0 = (n * w / waves) & ~INT64_C(3), b1 = w + 1 == waves ? n : (n * (w + 1) / waves) & ~INT64_C(3);
+        const int64_t m = b1 - b0;
+        const int32_t *list = g->bin_list[0] + b0;
+        const int grid = bulk ? grid_for((m + 3) / 4, kThreadThreads, num_sms() * 8)   // 4 entries per thread and step
+                              : grid_for(m, kThreadThreads, num_sms() * 32);
+        if (md <= 4)
+            k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+        else if (md <= 8)
+            k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+        else if (md <= 16)
+            k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+        else
+            k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+        CU(cudaGetLastError());
+    }
+    g->stats.launches[0] += (int)waves - 1;
     return NULPA_OK;
 }
 
@@ -1996,11 +2080,14 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             WarpSched ws{sched_block == 0 ? SCHED_STEAL : sched_block == 1 ? SCHED_STRIDED : SCHED_GUIDED,
                          sched_block, ctr + kCtrSchedW, g->wranges};
             int grid = sms * kWarpCtasPerSm;
-            if (ws.mode == SCHED_STEAL) {
+            if (ws.mode == SCHED_STEAL && g->locality >= kLocalRuns) {
                 // each warp walks one run of bin / warps rows; on a small bin
-                // (a test graph, a row shard of a multi-GPU run) launch only
-                // enough warps for runs of >= kMinFirstRun rows (modularity:
-                // labels propagate along ID order within a run)
+                // (a test graph, a row shard of a multi-GPU run) whose IDs
+                // carry locality (web crawls in URL order, road networks)
+                // launch only enough warps for runs of >= kMinFirstRun rows
+                // (modularity: labels propagate along ID order within a run;
+                // DESIGN.md "Quality notes").  Without ID locality (permuted
+                // SBM / R-MAT IDs) runs buy nothing: full grid.
                 ws.K = (int)(kMinFirstRun / 32);
                 const int64_t warps = std::max<int64_t>(1, n / kMinFirstRun);
                 grid = (int)std::min<int64_t>(grid, (warps + kWarpWarps - 1) / kWarpWarps);
@@ -2354,12 +2441,17 @@ int nulpa_run(nulpa_graph *g, const nulpa_params *params, nulpa_stats *stats) {
             s.edges_scanned[b] += (int64_t)c[5 + b];
             s.vertices_changed[b] += (int64_t)c[9 + b];
             s.changed_edges[b] += (int64_t)c[13 + b];
+            s.iter_processed[it][b] = (int64_t)c[1 + b];
+            s.iter_edges[it][b] = (int64_t)c[5 + b];
+            s.iter_changed[it][b] = (int64_t)c[9 + b];
+            s.iter_changed_edges[it][b] = (int64_t)c[13 + b];
         }
         if (timing) {
             for (int b = 0; b < 4; ++b) {
                 float ms = 0;
                 CU(cudaEventElapsedTime(&ms, g->ev[(it * 4 + b) * 2], g->ev[(it * 4 + b) * 2 + 1]));
                 s.kernel_ms[b] += ms;
+                s.iter_kernel_ms[it][b] = ms;
             }
         }
     }

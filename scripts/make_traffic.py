@@ -1,9 +1,23 @@
-"""profiles/traffic.json from an ncu launch list with dram__bytes_read/write
+"""Merge DRAM traffic per sweep of one degree bin into profiles/traffic.json.
+
+Input: an ncu launch list with dram__bytes_read/write of one nu-LPA run
 (`ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum
--k regex:^k_ --csv --log-file X python bench.py ...`): DRAM bytes per sweep of
-the warp bin (one k_frontier + one k_warp launch per sweep)."""
-import csv, collections, json, sys
-path, workload, weights = sys.argv[1], sys.argv[2], sys.argv[3]
+--clock-control none --csv --log-file X python scripts/profile_run.py --config C --runs 1`).
+
+    python scripts/make_traffic.py X <config> <weights> warp|thread
+
+warp bin of a sweep = the k_frontier launch right before each k_warp<..., 512,
+...> launch; thread bin = each k_thread launch.  The bench reads
+traffic.json["<config>/<weights>/<bin>"]["dram_bytes_per_sweep"] as the
+roofline's `traffic` (same per-sweep unit as algorithmic_bytes_per_sweep).
+"""
+import collections
+import csv
+import json
+import os
+import sys
+
+path, config, weights, binname = sys.argv[1:5]
 rows = [r for r in csv.reader(open(path)) if r]
 hi = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
 h = rows[hi]
@@ -15,17 +29,32 @@ for r in rows[hi + 1:]:
         continue
     per[r[iid]][r[im]] = float(r[iv].replace(",", ""))
     name[r[iid]] = r[ik]
+
+
 def dram(k):
     return per[k]["dram__bytes_read.sum"] + per[k]["dram__bytes_write.sum"]
+
+
 ids = sorted(per, key=int)
-# the warp bin of a sweep = the k_frontier launch right before each k_warp<..., 512> launch
-warp = [k for k in ids if "k_warp" in name[k] and "512>" in name[k]]
-front = [ids[ids.index(k) - 1] for k in warp]
-assert all("k_frontier" in name[f] for f in front)
-b = [dram(f) + dram(w) for f, w in zip(front, warp)]
-out = {"workload": workload, "weights": weights, "bin": "warp", "kernels": ["k_frontier", "k_warp"],
-       "sweeps": len(b), "dram_bytes_per_sweep": sum(b) / len(b), "per_sweep": b,
-       "k_warp_per_launch": [dram(w) for w in warp], "k_frontier_per_launch": [dram(f) for f in front],
-       "source": path, "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none (cold, serialised launches)"}
-json.dump(out, open("profiles/traffic.json", "w"), indent=1)
-print(out["dram_bytes_per_sweep"] / 1e9, "GB per sweep over", len(b), "sweeps")
+if binname == "warp":
+    main = [k for k in ids if "k_warp" in name[k] and ", 512" in name[k]]
+    front = [ids[ids.index(k) - 1] for k in main]
+    assert all("k_frontier" in name[f] for f in front), [name[f] for f in front]
+    b = [dram(f) + dram(w) for f, w in zip(front, main)]
+    kernels = ["k_frontier", "k_warp"]
+    extra = {"k_warp_per_launch": [dram(w) for w in main], "k_frontier_per_launch": [dram(f) for f in front]}
+else:
+    main = [k for k in ids if "k_thread" in name[k]]
+    b = [dram(k) for k in main]
+    kernels = ["k_thread"]
+    extra = {}
+out_path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "traffic.json")
+db = json.load(open(out_path)) if os.path.exists(out_path) else {}
+if "workload" in db:          # round-1 single-entry format
+    db = {}
+db[f"{config}/{weights}/{binname}"] = {
+    "kernels": kernels, "sweeps": len(b), "dram_bytes_per_sweep": sum(b) / len(b), "per_sweep": b, **extra,
+    "source": os.path.basename(path),
+    "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none (cold, serialised launches)"}
+json.dump(db, open(out_path, "w"), indent=1)
+print(config, binname, sum(b) / len(b) / 1e9, "GB per sweep over", len(b), "sweeps")
