@@ -49,8 +49,7 @@ constexpr int kCtrSchedW = 17;           // counter slot: dynamic schedule of th
 constexpr int kCtrSchedB = 18;           // counter slot: dynamic schedule of the wide k_warp
 // counter slots: 0 dN, 1+b processed, 5+b edges, 9+b changed, 13+b edges of changed (b = bin)
 
-constexpr int kBlockThreads = 512;       // k_block / giant kernels
-constexpr int kBlockCap = 4096;          // slots per CTA table (degree <= 4095 -> p1 <= 4095)
+constexpr int kBlockThreads = 512;       // giant kernels
 constexpr int kGiantChunk = 2048;        // edges per giant chunk
 constexpr int kGiantCap = 4096;          // slots of a chunk table (2048 edges -> p1 = 4095)
 constexpr int kThreadThreads = 256;
@@ -1018,133 +1017,159 @@ done:
 }
 
 // ---------------------------------------------------------------------------
-// block-per-vertex kernel: one CTA of 4 warps per vertex, the
-// vertex's table -- p1 = nextPow2(D)-1 slots as in PAPER.md:208, <= 4095 --
-// in shared memory, cleared at the start of each vertex.  Each warp folds its
-// 32-edge batches (match_any groups); a group leader claims the label's slot
-// (Algorithm 2 probing, atomicCAS) and adds the group total with one
-// atomicAdd, whose return value gives the label's running total, so the
-// maximum over all leaders' totals is hashtableMaxKey (no table scan).
+// block-per-vertex kernel: one CTA of 8 warps per vertex
+// (degree wide_degree <= D < giant_degree), the vertex's table -- p1 =
+// nextPow2(D)-1 slots as in PAPER.md:208 -- in shared memory.  The row is
+// staged by TMA: one thread issues a 1-D bulk copy (cp.async.bulk, mbarrier
+// completion) of the NEXT vertex's indices (and weights) into the other of
+// two shared row buffers while the CTA folds this one, so no thread waits
+// on a dependent CSR load; all label gathers C[j] of a row are issued
+// before its fold (up to R per thread, in registers).  Per 32-entry batch a
+// warp folds equal labels with match_any; the group leader claims the
+// label's slot (Algorithm 2 probing, atomicCAS) and adds the group total --
+// an integer count (exact for unit weights, native shared atomicAdd) or,
+// for other weights, a float atomicAdd.  hashtableMaxKey is a scan of the
+// table's p1 slots (ties: smallest label, R6).
 // ---------------------------------------------------------------------------
-constexpr int kBlkThreads = 128;
+constexpr int kBlkThreads = 256;
 
-template <bool SYNC, bool W>
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(bar), "r"(parity) : "memory");
+}
+// 1-D bulk copy global -> shared (TMA), completion counted on mbarrier `bar`
+__device__ __forceinline__ void tma_load_1d(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+// R: label gathers per thread (rows of up to R * kBlkThreads entries);
+// rowcap: entries per row buffer (>= max degree + 4, multiple of 4);
+// cap: table slots (>= p1 of the largest degree).
+template <bool SYNC, bool W, int R>
 __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *__restrict__ recs,
-                                                        const unsigned long long *__restrict__ count) {
-    extern __shared__ int32_t dyn[];
-    int32_t *Hk = dyn;
-    float *Hv = reinterpret_cast<float *>(dyn + kBlockCap);
-    __shared__ int64_t m_o[32];
-    __shared__ int32_t m_r[32], m_d[32], m_ci[32];
-    __shared__ unsigned s_act;
+                                                        const unsigned long long *__restrict__ count, int cap,
+                                                        int rowcap) {
+    extern __shared__ __align__(16) uint8_t dyn_b[];
+    int32_t *Hk = reinterpret_cast<int32_t *>(dyn_b);                 // keys (kEmpty = free)
+    uint32_t *Hc = reinterpret_cast<uint32_t *>(Hk + cap);            // unit-weight counts
+    float *Hf = reinterpret_cast<float *>(Hc + cap);                  // other weights
+    int32_t *rowi = reinterpret_cast<int32_t *>(Hf + cap);            // 2 index buffers of rowcap
+    float *roww = reinterpret_cast<float *>(rowi + 2 * rowcap);       // 2 weight buffers (W)
+    __shared__ __align__(8) uint64_t s_bar[2];
+    __shared__ uint64_t s_best[kBlkThreads / 32];
     __shared__ int s_changed;
-    __shared__ uint32_t s_bw[kBlkThreads / 32], s_rr[kBlkThreads / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    unsigned long long n_changed = 0, n_changed_edges = 0;
+    const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(&s_bar[0]);
     const int64_t n = (int64_t)*count;
-    const int64_t ngroups = (n + 31) / 32;
-    for (int64_t gq = blockIdx.x; gq < ngroups; gq += gridDim.x) {
-        // 32 frontier records (k_frontier: unprocessed vertices, flags already cleared)
-        if (wid == 0) {
-            const int64_t t = gq * 32 + lane;
-            if (t < n) {
-                const VRec rc = recs[t];
-                m_o[lane] = (int64_t)(((uint64_t)(rc.o_hi_deg & 0xFFFFu) << 32) | rc.o_lo);
-                m_d[lane] = (int32_t)(rc.o_hi_deg >> 16);
-                m_r[lane] = rc.r;
-                m_ci[lane] = rc.ci;
+    unsigned long long n_changed = 0, n_changed_edges = 0;
+    auto r_o = [](const VRec &r) -> int64_t { return (int64_t)(((uint64_t)(r.o_hi_deg & 0xFFFFu) << 32) | r.o_lo); };
+    auto r_d = [](const VRec &r) -> uint32_t { return r.o_hi_deg >> 16; };
+    // the row of record r into buffer b (one thread): indices [o & ~3, ...)
+    auto stage = [&](const VRec &r, int b) {
+        const int64_t o = r_o(r), o0 = o & ~INT64_C(3);
+        const uint32_t ents = (uint32_t)(((o + r_d(r) - o0) + 3) & ~INT64_C(3));
+        const uint32_t bar = bar0 + 8u * b;
+        mbar_expect_tx(bar, ents * 4u * (W ? 2u : 1u));
+        tma_load_1d((uint32_t)__cvta_generic_to_shared(rowi + b * rowcap), a.indices + o0, ents * 4u, bar);
+        if (W) tma_load_1d((uint32_t)__cvta_generic_to_shared(roww + b * rowcap), a.weights + o0, ents * 4u, bar);
+    };
+    if (threadIdx.x == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar0 + 8, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && (int64_t)blockIdx.x < n) stage(recs[blockIdx.x], 0);
+    int i = 0;
+    for (int64_t k = blockIdx.x; k < n; k += gridDim.x, ++i) {
+        const int b = i & 1;
+        const VRec rc = recs[k];
+        if (threadIdx.x == 0 && k + gridDim.x < n) {
+            // buffer b^1 was last read by vertex i-1 (done: trailing __syncthreads)
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            stage(recs[k + gridDim.x], b ^ 1);
+        }
+        const uint32_t deg = r_d(rc);
+        const int64_t v = rc.r + a.row_begin;
+        Hash h;
+        h.init(deg);
+        for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {   // hashtableClear
+            Hk[q] = kEmpty;
+            Hc[q] = 0;
+            Hf[q] = 0.0f;
+        }
+        mbar_wait(bar0 + 8u * b, (uint32_t)(i >> 1) & 1u);
+        const int32_t *ri = rowi + b * rowcap + (r_o(rc) & 3);
+        const float *rw = roww + b * rowcap + (r_o(rc) & 3);
+        // every label gather of the row in flight at once
+        int32_t key[R];
+        float w[R];
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+            const uint32_t e = (uint32_t)(u * kBlkThreads) + threadIdx.x;
+            key[u] = kEmpty;
+            w[u] = 1.0f;
+            if (e < deg) {
+                const int32_t j = ri[e];
+                if (j != (int32_t)v) key[u] = a.lab_in[j];          // "if j = i continue"
+                if (W) w[u] = rw[e];
             }
-            const unsigned am = __ballot_sync(0xFFFFFFFFu, t < n);
-            if (lane == 0) s_act = am;
+        }
+        __syncthreads();                                             // table cleared
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+            if ((uint32_t)(u * kBlkThreads) + (uint32_t)(wid * 32) >= deg) break;   // warp-uniform
+            const unsigned grp = __match_any_sync(0xFFFFFFFFu, key[u]);
+            const bool leader = key[u] != kEmpty && (grp & ((1u << lane) - 1)) == 0;
+            const bool eq = !W || __all_sync(0xFFFFFFFFu, key[u] == kEmpty || w[u] == 1.0f);
+            float x = 0.0f;
+            if (!eq) {
+                const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key[u] != kEmpty ? (unsigned)__popc(grp) : 1u);
+                x = maxn > 1 ? group_sum(grp, w[u], maxn) : w[u];
+            }
+            if (leader) {
+                const uint32_t slot = ht_claim(Hk, h, key[u]);
+                if (eq) atomicAdd(&Hc[slot], (uint32_t)__popc(grp));
+                else atomicAdd(&Hf[slot], x);
+            }
+        }
+        __syncthreads();                                             // table complete
+        // hashtableMaxKey: (total, smallest label) as one 64-bit max
+        uint64_t best = 0;
+        for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {
+            const int32_t kk = Hk[q];
+            if (kk == kEmpty) continue;
+            const float t = __fadd_rn((float)Hc[q], Hf[q]);
+            const uint64_t c = ((uint64_t)(__float_as_uint(t) + 1) << 32) | (uint32_t)~kk;
+            best = c > best ? c : best;
+        }
+        best = warp_max_u64(best);
+        if (lane == 0) s_best[wid] = best;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint64_t bb = 0;
+            for (int q = 0; q < kBlkThreads / 32; ++q) bb = s_best[q] > bb ? s_best[q] : bb;
+            const int32_t cs = bb ? (int32_t)~(uint32_t)bb : kEmpty;
+            const int ch = accept_move(cs, rc.ci, a.pickless);
+            if (ch) a.lab_out[v] = cs;
+            s_changed = ch;
+            n_changed += ch;
+            n_changed_edges += ch ? deg : 0;
         }
         __syncthreads();
-        unsigned act = s_act;
-        while (act) {
-            const int k = __ffs(act) - 1;
-            act &= act - 1;
-            const int64_t o = m_o[k];
-            const uint32_t deg = (uint32_t)m_d[k];
-            const int64_t v = m_r[k] + a.row_begin;
-            Hash h;
-            h.init(deg);
-            for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {   // hashtableClear
-                Hk[q] = kEmpty;
-                Hv[q] = 0.0f;
-            }
-            __syncthreads();
-            TieOrder to;
-            to.init(h);
-            uint32_t bw = 0;
-            int32_t bk = 0;
-            auto fold = [&](int32_t key, float w) {
-                const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
-                float x;
-                if (W) {
-                    const float w_ref = __shfl_sync(0xFFFFFFFFu, w, 0);
-                    if (__all_sync(0xFFFFFFFFu, key == kEmpty || w == w_ref)) {
-                        x = (float)__popc(grp) * w;
-                    } else {
-                        const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key != kEmpty ? (unsigned)__popc(grp) : 1u);
-                        x = maxn > 1 ? group_sum(grp, w, maxn) : w;
-                    }
-                } else {
-                    x = (float)__popc(grp);
-                }
-                if (key != kEmpty && lane == __ffs(grp) - 1) {
-                    const uint32_t slot = ht_claim(Hk, h, key);
-                    const float V = __fadd_rn(atomicAdd(&Hv[slot], x), x);
-                    const uint32_t vb = __float_as_uint(V) + 1;
-                    if (vb > bw || (vb == bw && to.rank(key) < to.rank(bk))) {
-                        bw = vb;
-                        bk = key;
-                    }
-                }
-            };
-            // two 32-edge batches per warp per step: both index loads, then
-            // both label gathers in flight together
-            for (uint32_t b = (uint32_t)wid * 32; b < deg; b += 2 * kBlkThreads) {
-                const uint32_t e0 = b + lane, e1 = b + kBlkThreads + lane;
-                const int32_t j0 = e0 < deg ? ld_stream(a.indices + o + e0) : -1;
-                const int32_t j1 = e1 < deg ? ld_stream(a.indices + o + e1) : -1;
-                float w0 = 0.0f, w1 = 0.0f;
-                if (W) {
-                    if (e0 < deg) w0 = ld_stream(a.weights + o + e0);
-                    if (e1 < deg) w1 = ld_stream(a.weights + o + e1);
-                }
-                const int32_t k0 = (j0 >= 0 && j0 != (int32_t)v) ? a.lab_in[j0] : kEmpty;   // "if j = i continue"
-                const int32_t k1 = (j1 >= 0 && j1 != (int32_t)v) ? a.lab_in[j1] : kEmpty;
-                fold(k0, w0);
-                if (b + kBlkThreads < deg) fold(k1, w1);
-            }
-            // hashtableMaxKey over the 4 warps
-            const uint32_t W1 = __reduce_max_sync(0xFFFFFFFFu, bw);
-            const uint32_t rr = (bw == W1 && W1) ? 0xFFFFFFFFu - to.rank(bk) : 0u;
-            const uint32_t R1 = __reduce_max_sync(0xFFFFFFFFu, rr);
-            if (lane == 0) {
-                s_bw[wid] = W1;
-                s_rr[wid] = R1;
-            }
-            __syncthreads();
-            if (threadIdx.x == 0) {
-                uint32_t Wb = 0, Rb = 0;
-                for (int q = 0; q < kBlkThreads / 32; ++q) {
-                    if (s_bw[q] > Wb || (s_bw[q] == Wb && s_rr[q] > Rb)) {
-                        Wb = s_bw[q];
-                        Rb = s_rr[q];
-                    }
-                }
-                const int32_t cs = Wb ? to.unrank(0xFFFFFFFFu - Rb) : kEmpty;
-                const int ch = accept_move(cs, m_ci[k], a.pickless);
-                if (ch) a.lab_out[v] = cs;
-                s_changed = ch;
-                n_changed += ch;
-                n_changed_edges += ch ? deg : 0;
-            }
-            __syncthreads();
-            if (s_changed)
-                for (uint32_t b = threadIdx.x; b < deg; b += kBlkThreads) a.flag_out[a.indices[o + b]] = 1;
-        }
-        __syncthreads();
+        if (s_changed)
+            for (uint32_t e = threadIdx.x; e < deg; e += kBlkThreads) a.flag_out[ri[e]] = 1;
+        __syncthreads();                                             // row buffer b and s_changed reusable
     }
     if (threadIdx.x == 0 && n_changed) {
         atomicAdd(&a.ctr[0], n_changed);
@@ -2059,9 +2084,21 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                     k_warp<SYNC, W, kWideSlots, false><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
                 g->stats.launches[2] += 1;
             }
-            const size_t smem = kBlockCap * (sizeof(int32_t) + sizeof(float));
-            k_block<SYNC, W><<<grid_for((n + 31) / 32, 1, sms * 7), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB);
-            CU(cudaGetLastError());
+            // k_block: table of the largest p1, two TMA row buffers
+            const int maxdeg = std::max(1, p.giant_degree - 1);
+            const int cap = (int)capacity_p1((uint32_t)maxdeg) + 1;
+            const int rowcap = (maxdeg + 4 + 3) & ~3;
+            const size_t smem = (size_t)cap * 12 + (size_t)rowcap * 4 * 2 * (W ? 2 : 1);
+            auto launch_block = [&](auto kern) -> int {
+                CU(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                int per_sm = 0;
+                CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlkThreads, smem));
+                kern<<<grid_for(n, 1, sms * std::max(1, per_sm)), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB, cap, rowcap);
+                CU(cudaGetLastError());
+                return NULPA_OK;
+            };
+            if (maxdeg + 3 <= 8 * kBlkThreads) CHECK(launch_block(k_block<SYNC, W, 8>));
+            else CHECK(launch_block(k_block<SYNC, W, 16>));
             g->stats.launches[2] += 2;
         }
         CHECK(rec(2, 1));
