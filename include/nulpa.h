@@ -194,6 +194,28 @@ int nulpa_modularity_partial(nulpa_graph *g, const int32_t *labels_device, doubl
 int nulpa_modularity_finish(nulpa_graph *g, const double *Sigma_device, double sigma_intra,
                             double two_m, double *q);
 
+/* Multi-GPU exchange primitives (distributed.py; the bulk-synchronous
+ * label / mark exchange after every lpaMove of a row shard, north star
+ * "changed labels are exchanged per iteration").  All pointers are device
+ * memory; work is enqueued on the handle's stream.
+ *
+ * nulpa_pack_changed: for every row r of this shard whose current label
+ * differs from prev_device[r] (the shard's labels saved before the sweep,
+ * n_rows int32), write one pair (vertex << 32) | label into pairs_device
+ * (capacity n_rows int64; order arbitrary); *count = pairs written
+ * (synchronises the stream). */
+int nulpa_pack_changed(nulpa_graph *g, const int32_t *prev_device, long long *pairs_device, int64_t *count);
+/* Apply n pairs to the label vector (pairs < 0 are padding, skipped). */
+int nulpa_apply_pairs(nulpa_graph *g, const long long *pairs_device, int64_t n);
+/* Pack the unprocessed flags of every rank's row range q = [bounds[q],
+ * bounds[q+1]) (bounds_device: P+1 int64) into bits_device[q*words ..]
+ * (words uint32 per range, bit t of word w = flag of row bounds[q]+32w+t),
+ * then clear the flags outside this shard's rows. */
+int nulpa_pack_flag_bits(nulpa_graph *g, const int64_t *bounds_device, int P, int64_t words, uint32_t *bits_device);
+/* This shard's flags = OR over P received bitmaps of its own range
+ * (bits_device: P*words uint32, words*32 >= n_rows). */
+int nulpa_or_flag_bits(nulpa_graph *g, const uint32_t *bits_device, int P, int64_t words);
+
 int nulpa_get_stats(nulpa_graph *g, nulpa_stats *out);
 
 /* Return the device memory that destroyed handles left in the library's

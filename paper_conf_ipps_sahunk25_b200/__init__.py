@@ -20,7 +20,8 @@ __all__ = [
     "NulpaError", "Params", "Stats", "Graph", "lpa", "load_library", "library_path",
     "nulpa_create", "nulpa_run", "nulpa_sweep", "nulpa_labels", "nulpa_set_labels", "nulpa_flags",
     "nulpa_modularity", "nulpa_modularity_partial", "nulpa_modularity_finish", "nulpa_reset",
-    "nulpa_bind_state", "nulpa_get_stats", "nulpa_release_memory", "nulpa_destroy", "nulpa_default_params", "nulpa_version",
+    "nulpa_bind_state", "nulpa_get_stats", "nulpa_release_memory", "nulpa_pack_changed", "nulpa_apply_pairs",
+    "nulpa_pack_flag_bits", "nulpa_or_flag_bits", "nulpa_destroy", "nulpa_default_params", "nulpa_version",
     "ASYNC", "SYNC", "MEM_HOST", "MEM_DEVICE",
 ]
 
@@ -131,6 +132,10 @@ def load_library():
         "nulpa_state_pointers": (ctypes.c_int, [vp, P(vp), P(vp)]),
         "nulpa_destroy": (ctypes.c_int, [vp]),
         "nulpa_release_memory": (ctypes.c_int, []),
+        "nulpa_pack_changed": (ctypes.c_int, [vp, vp, vp, P(i64)]),
+        "nulpa_apply_pairs": (ctypes.c_int, [vp, vp, i64]),
+        "nulpa_pack_flag_bits": (ctypes.c_int, [vp, vp, ctypes.c_int, i64, vp]),
+        "nulpa_or_flag_bits": (ctypes.c_int, [vp, vp, ctypes.c_int, i64]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -252,6 +257,24 @@ def nulpa_bind_state(h, labels_device, flags_device):
 def nulpa_release_memory():
     """Return pooled device memory of destroyed handles to the driver."""
     _check(load_library().nulpa_release_memory())
+
+
+def nulpa_pack_changed(h, prev_device, pairs_device) -> int:
+    n = ctypes.c_int64(0)
+    _check(load_library().nulpa_pack_changed(h, _ptr(prev_device), _ptr(pairs_device), ctypes.byref(n)))
+    return n.value
+
+
+def nulpa_apply_pairs(h, pairs_device, n: int):
+    _check(load_library().nulpa_apply_pairs(h, _ptr(pairs_device), int(n)))
+
+
+def nulpa_pack_flag_bits(h, bounds_device, P: int, words: int, bits_device):
+    _check(load_library().nulpa_pack_flag_bits(h, _ptr(bounds_device), int(P), int(words), _ptr(bits_device)))
+
+
+def nulpa_or_flag_bits(h, bits_device, P: int, words: int):
+    _check(load_library().nulpa_or_flag_bits(h, _ptr(bits_device), int(P), int(words)))
 
 
 def nulpa_get_stats(h) -> Stats:

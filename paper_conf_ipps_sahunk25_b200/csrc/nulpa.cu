@@ -1804,6 +1804,66 @@ void free_bins(nulpa_graph *g) {
     g->bins_built = false;
 }
 
+// ---------------------------------------------------------------------------
+// multi-GPU exchange (distributed.py): changed labels as (vertex, label)
+// pairs, marks as per-rank bitmaps
+// ---------------------------------------------------------------------------
+// pairs[k] = vertex << 32 | label for every own row whose label differs from
+// prev (the rank's labels before the sweep); *cnt = number of pairs
+// (warp-aggregated atomics; pair order is arbitrary, vertices are unique)
+__global__ void k_pack_changed(const int32_t *__restrict__ lab, const int32_t *__restrict__ prev, int64_t row_begin,
+                               int64_t n, long long *pairs, unsigned long long *cnt) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = base + threadIdx.x;
+        const int32_t c = r < n ? lab[row_begin + r] : 0;
+        const bool ch = r < n && c != prev[r];
+        const unsigned m = __ballot_sync(0xFFFFFFFFu, ch);
+        if (!m) continue;
+        unsigned long long pos = 0;
+        if (lane == 0) pos = atomicAdd(cnt, (unsigned long long)__popc(m));
+        pos = __shfl_sync(0xFFFFFFFFu, pos, 0) + __popc(m & ((1u << lane) - 1));
+        if (ch) pairs[pos] = (long long)(((uint64_t)(row_begin + r) << 32) | (uint32_t)c);
+    }
+}
+// lab[vertex] = label for every pair (pairs < 0 are padding)
+__global__ void k_apply_pairs(int32_t *lab, const long long *__restrict__ pairs, int64_t n) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
+        const long long p = pairs[k];
+        if (p >= 0) lab[(int64_t)((uint64_t)p >> 32)] = (int32_t)(uint32_t)p;
+    }
+}
+// bits[q][w] bit t = flags[bounds[q] + 32w + t] for every rank range q
+// (words words per range); afterwards the flags outside [own_b, own_e) are
+// cleared (each rank keeps only its own rows' marks)
+__global__ void k_pack_flag_bits(uint8_t *flags, const int64_t *__restrict__ bounds, int P, int64_t words,
+                                 uint32_t *bits, int64_t own_b, int64_t own_e) {
+    const int64_t tot = (int64_t)P * words;
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < tot; k += (int64_t)gridDim.x * blockDim.x) {
+        const int q = (int)(k / words);
+        const int64_t w = k - (int64_t)q * words, b = bounds[q], e = bounds[q + 1];
+        uint32_t x = 0;
+        for (int t = 0; t < 32; ++t) {
+            const int64_t i = b + 32 * w + t;
+            if (i < e && flags[i]) x |= 1u << t;
+        }
+        bits[k] = x;
+    }
+}
+__global__ void k_clear_remote_flags(uint8_t *flags, int64_t n, int64_t own_b, int64_t own_e) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (i < own_b || i >= own_e) flags[i] = 0;
+}
+// flags[own_b + i] = OR over the P ranks' bitmaps of the own range
+__global__ void k_or_flag_bits(uint8_t *flags, const uint32_t *__restrict__ bits, int P, int64_t words, int64_t own_b,
+                               int64_t own_e) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; own_b + i < own_e; i += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t x = 0;
+        for (int q = 0; q < P; ++q) x |= bits[(int64_t)q * words + (i >> 5)];
+        flags[own_b + i] = (x >> (i & 31)) & 1u;
+    }
+}
+
 __global__ void k_fill_i32(int32_t *p, int64_t n, int32_t v) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
 }
@@ -2397,6 +2457,56 @@ int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *we
     nulpa_default_params(&p);
     if ((r = build_bins(g, p.switch_degree, p.block_degree, p.giant_degree))) return bail(r);
     *out = g;
+    return NULPA_OK;
+}
+
+int nulpa_pack_changed(nulpa_graph *g, const int32_t *prev_device, long long *pairs_device, int64_t *count) {
+    if (!g || !prev_device || !pairs_device || !count) return fail(NULPA_EINVAL, "null argument");
+    unsigned long long *cnt = g->ctr + (size_t)kMaxIter * kCtr + kCtr - 1;
+    CU(cudaMemsetAsync(cnt, 0, sizeof *cnt, g->stream));
+    if (g->n_rows > 0) {
+        k_pack_changed<<<grid_for(g->n_rows, 256, num_sms() * 8), 256, 0, g->stream>>>(g->labels, prev_device, g->row_begin,
+                                                                                     g->n_rows, pairs_device, cnt);
+        CU(cudaGetLastError());
+    }
+    unsigned long long h = 0;
+    CU(cudaMemcpyAsync(&h, cnt, sizeof h, cudaMemcpyDeviceToHost, g->stream));
+    CU(cudaStreamSynchronize(g->stream));
+    *count = (int64_t)h;
+    return NULPA_OK;
+}
+
+int nulpa_apply_pairs(nulpa_graph *g, const long long *pairs_device, int64_t n) {
+    if (!g || (n > 0 && !pairs_device)) return fail(NULPA_EINVAL, "null argument");
+    if (n > 0) {
+        k_apply_pairs<<<grid_for(n, 256, num_sms() * 8), 256, 0, g->stream>>>(g->labels, pairs_device, n);
+        CU(cudaGetLastError());
+    }
+    return NULPA_OK;
+}
+
+int nulpa_pack_flag_bits(nulpa_graph *g, const int64_t *bounds_device, int P, int64_t words, uint32_t *bits_device) {
+    if (!g || !bounds_device || !bits_device || P < 1 || words < 0) return fail(NULPA_EINVAL, "bad argument");
+    const int64_t tot = (int64_t)P * words;
+    if (tot > 0) {
+        k_pack_flag_bits<<<grid_for(tot, 256, num_sms() * 8), 256, 0, g->stream>>>(g->flags, bounds_device, P, words,
+                                                                                 bits_device, g->row_begin,
+                                                                                 g->row_begin + g->n_rows);
+        CU(cudaGetLastError());
+    }
+    k_clear_remote_flags<<<grid_for(g->n_global, 256, num_sms() * 8), 256, 0, g->stream>>>(g->flags, g->n_global, g->row_begin,
+                                                                                        g->row_begin + g->n_rows);
+    CU(cudaGetLastError());
+    return NULPA_OK;
+}
+
+int nulpa_or_flag_bits(nulpa_graph *g, const uint32_t *bits_device, int P, int64_t words) {
+    if (!g || !bits_device || P < 1 || words * 32 < g->n_rows) return fail(NULPA_EINVAL, "bad argument");
+    if (g->n_rows > 0) {
+        k_or_flag_bits<<<grid_for(g->n_rows, 256, num_sms() * 8), 256, 0, g->stream>>>(g->flags, bits_device, P, words,
+                                                                                     g->row_begin, g->row_begin + g->n_rows);
+        CU(cudaGetLastError());
+    }
     return NULPA_OK;
 }
 

@@ -6,21 +6,30 @@ is split into contiguous ranges holding ~|E|/P CSR entries each
 lpaMove, through ``nulpa_sweep`` on a shard handle)
 against a REPLICATED label vector, then
 
-  * the labels of every rank's range are exchanged with an all-gather
-    (``all_gather_into_tensor`` over a padded [P, max_rows] staging buffer);
-  * the "unprocessed" marks a rank set on other ranks' vertices are merged
-    with a reduce-scatter(MAX) over the same padded layout: each rank
-    receives the maximum of everybody's marks for its own rows only;
-  * dN is all-reduced (SUM) and Algorithm 1's tolerance / Pick-Less loop
-     runs identically on every rank.
+  * only CHANGED labels travel: each rank packs its rows whose label moved
+    in this sweep as (vertex, label) pairs (``nulpa_pack_changed``), the
+    per-rank counts are all-gathered (their sum is dN), and the pairs are
+    all-gathered over a [P, max count] buffer and applied
+    (``nulpa_apply_pairs``) -- 8 bytes per changed vertex instead of 4 per
+    vertex.  When more than 1/8 of all vertices changed (the first sweeps)
+    the label ranges are all-gathered densely instead (4 bytes per vertex,
+    ``all_gather_into_tensor`` over a padded [P, max_rows] buffer);
+  * the "unprocessed" marks a rank set are exchanged as bitmaps: per rank
+    range one bit per vertex (``nulpa_pack_flag_bits``), sent with one
+    all-to-all, OR-ed into the owner's flags (``nulpa_or_flag_bits``) --
+    N/8 bytes per rank instead of a byte per vertex;
+  * Algorithm 1's tolerance / Pick-Less loop runs
+    identically on every rank from the global dN.
 
 Within a rank the sweep is asynchronous (in-place labels); across ranks it
 is bulk-synchronous (remote labels are one sweep old).  The driver only
 moves tensors: all label computation happens in the CUDA kernels behind the
 C ABI (``CudaShardRunner``).  A runner is any object with ``N_global``,
 ``row_begin``, ``row_end``, ``labels`` (int32 [N]), ``flags`` (uint8 [N]),
-``reset()`` and ``sweep(pickless) -> int``, so the host logic can be tested
-with the gloo backend on CPU.
+``reset()``, ``sweep(pickless) -> int`` and the exchange primitives
+``snapshot()``, ``pack_changed(pairs) -> int``, ``apply_pairs(pairs, n)``,
+``pack_flag_bits(bounds, P, words, bits)``, ``or_flag_bits(bits, P, words)``,
+so the host logic can be tested with the gloo backend on CPU.
 """
 from __future__ import annotations
 
@@ -96,6 +105,24 @@ class CudaShardRunner:
     def sweep(self, pickless: bool) -> int:
         return self.nl.nulpa_sweep(self.g.h, pickless, self.params)
 
+    # exchange primitives (kernels behind the C ABI)
+    def snapshot(self):
+        if not hasattr(self, "prev"):
+            self.prev = torch.empty(max(1, self.row_end - self.row_begin), dtype=torch.int32, device=self.labels.device)
+        self.prev[: self.row_end - self.row_begin].copy_(self.labels[self.row_begin:self.row_end])
+
+    def pack_changed(self, pairs: torch.Tensor) -> int:
+        return self.nl.nulpa_pack_changed(self.g.h, self.prev, pairs)
+
+    def apply_pairs(self, pairs: torch.Tensor, n: int):
+        self.nl.nulpa_apply_pairs(self.g.h, pairs, n)
+
+    def pack_flag_bits(self, bounds: torch.Tensor, P: int, words: int, bits: torch.Tensor):
+        self.nl.nulpa_pack_flag_bits(self.g.h, bounds, P, words, bits)
+
+    def or_flag_bits(self, bits: torch.Tensor, P: int, words: int):
+        self.nl.nulpa_or_flag_bits(self.g.h, bits, P, words)
+
     def modularity_partial(self, Sigma: torch.Tensor):
         return self.nl.nulpa_modularity_partial(self.g.h, self.labels, Sigma)
 
@@ -104,28 +131,64 @@ class CudaShardRunner:
 
 
 class Exchanger:
-    """Per-sweep exchange of labels (all-gather) and flags (reduce-scatter
-    MAX: a rank needs only its own rows' flags, so each rank receives the
-    element-wise maximum of everybody's marks for its range -- half the bytes
-    of an all-reduce of the whole flag vector)."""
+    """Per-sweep exchange between the ranks (module docstring): changed
+    labels as pairs (dense all-gather of the label ranges when more than
+    `dense_above` of all vertices changed), marks as bitmaps (all-to-all),
+    dN from the all-gathered per-rank change counts.  `log` keeps, per
+    sweep, the label mode and the bytes each rank sent."""
 
-    def __init__(self, runner, group=None):
+    def __init__(self, runner, group=None, dense_above: float = 1.0 / 8.0):
         self.r = runner
         self.group = group
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         bounds = getattr(runner, "bounds", None) or runner.shard.bounds
         self.bounds = bounds
-        self.maxrows = max(e - b for b, e in bounds)
+        self.N = runner.N_global
+        self.maxrows = max(1, max(e - b for b, e in bounds))
+        self.dense_above = dense_above
         dev = runner.labels.device
+        self.dev = dev
         self.stage_in = torch.empty(self.maxrows, dtype=torch.int32, device=dev)
         self.stage_out = torch.empty(self.world * self.maxrows, dtype=torch.int32, device=dev)
-        self.fstage_in = torch.zeros(self.world * self.maxrows, dtype=torch.uint8, device=dev)
-        self.fstage_out = torch.empty(self.maxrows, dtype=torch.uint8, device=dev)
+        self.pairs = torch.empty(self.maxrows, dtype=torch.int64, device=dev)
+        self.words = (self.maxrows + 31) // 32
+        self.bits_out = torch.empty(self.world * self.words, dtype=torch.int32, device=dev)
+        self.bits_in = torch.empty(self.world * self.words, dtype=torch.int32, device=dev)
+        self.bounds_t = torch.tensor([b for b, _ in bounds] + [bounds[-1][1]], dtype=torch.int64, device=dev)
         b, e = bounds[self.rank]
         self.own = (b, e)
+        self.log = []
+
+    def before_sweep(self):
+        self.r.snapshot()
+
+    def exchange(self) -> int:
+        """After a sweep: labels, marks; returns the global dN."""
+        n_loc = self.r.pack_changed(self.pairs)
+        cnt = torch.tensor([n_loc], dtype=torch.int64, device=self.dev)
+        counts = torch.empty(self.world, dtype=torch.int64, device=self.dev)
+        dist.all_gather_into_tensor(counts, cnt, group=self.group)
+        counts = counts.tolist()
+        dn = int(sum(counts))
+        if dn > self.dense_above * self.N:
+            self.labels()
+            mode, sent = "dense", 4 * (self.own[1] - self.own[0])
+        else:
+            m = max(counts)
+            if m > 0:
+                self.pairs[n_loc:m].fill_(-1)                  # padding, skipped by apply
+                recv = torch.empty(self.world * m, dtype=torch.int64, device=self.dev)
+                dist.all_gather_into_tensor(recv, self.pairs[:m], group=self.group)
+                self.r.apply_pairs(recv, self.world * m)
+            mode, sent = "sparse", 8 * m
+        self.flags()
+        self.log.append({"dn": dn, "labels": mode, "label_bytes_sent": sent,
+                         "flag_bytes_sent": 4 * self.words * self.world})
+        return dn
 
     def labels(self):
+        """Dense: every rank's label range, all-gathered."""
         b, e = self.own
         self.stage_in[: e - b].copy_(self.r.labels[b:e])
         dist.all_gather_into_tensor(self.stage_out, self.stage_in, group=self.group)
@@ -134,24 +197,15 @@ class Exchanger:
                 self.r.labels[qb:qe].copy_(self.stage_out[q * self.maxrows: q * self.maxrows + (qe - qb)])
 
     def flags(self):
-        f = self.r.flags
-        for q, (qb, qe) in enumerate(self.bounds):
-            if qe > qb:
-                self.fstage_in[q * self.maxrows: q * self.maxrows + (qe - qb)].copy_(f[qb:qe])
-        dist.reduce_scatter_tensor(self.fstage_out, self.fstage_in, op=dist.ReduceOp.MAX, group=self.group)
-        b, e = self.own
-        f[b:e].copy_(self.fstage_out[: e - b])
-        self.clear_remote_flags()
+        """Marks of every rank range as bitmaps, all-to-all, OR-ed into the owner's flags."""
+        self.r.pack_flag_bits(self.bounds_t, self.world, self.words, self.bits_out)   # also clears remote flags
+        dist.all_to_all_single(self.bits_in, self.bits_out, group=self.group)
+        self.r.or_flag_bits(self.bits_in, self.world, self.words)
 
     def clear_remote_flags(self):
         b, e = self.own
         self.r.flags[:b].zero_()
         self.r.flags[e:].zero_()
-
-    def changed(self, dn_local: int) -> int:
-        t = torch.tensor([dn_local], dtype=torch.int64, device=self.r.labels.device)
-        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=self.group)
-        return int(t.item())
 
 
 def lpa_distributed(runner, tolerance: float = 0.05, max_iterations: int = 20, pickless_period: int = 4,
@@ -168,16 +222,16 @@ def lpa_distributed(runner, tolerance: float = 0.05, max_iterations: int = 20, p
     launches = 0
     for l in range(max_iterations):
         pl = pickless_period > 0 and l % pickless_period == 0
-        dn_local = runner.sweep(pl)
-        ex.labels()
-        ex.flags()
-        dn = ex.changed(dn_local)
+        ex.before_sweep()
+        runner.sweep(pl)
+        dn = ex.exchange()
         changed.append(dn)
         launches += 1
         if not pl and dn / N < tolerance:
             converged = True
             break
-    return {"iterations": len(changed), "changed": changed, "converged": converged, "launches": launches}
+    return {"iterations": len(changed), "changed": changed, "converged": converged, "launches": launches,
+            "exchange": ex.log[-len(changed):]}
 
 
 def modularity_distributed(runner, group=None) -> float:

@@ -32,6 +32,43 @@ class OracleShardRunner:
         self.labels.copy_(torch.arange(self.N_global, dtype=torch.int32))
         self.flags.fill_(1)
 
+    # exchange primitives (reference semantics of the CUDA kernels behind
+    # nulpa_pack_changed / nulpa_apply_pairs / nulpa_pack_flag_bits /
+    # nulpa_or_flag_bits)
+    def snapshot(self):
+        self.prev = self.labels[self.row_begin:self.row_end].clone()
+
+    def pack_changed(self, pairs):
+        cur = self.labels[self.row_begin:self.row_end]
+        idx = torch.nonzero(cur != self.prev).flatten()
+        k = idx.numel()
+        pairs[:k] = ((idx + self.row_begin).to(torch.int64) << 32) | cur[idx].to(torch.int64)
+        return k
+
+    def apply_pairs(self, pairs, n):
+        p = pairs[:n]
+        p = p[p >= 0]
+        self.labels[p >> 32] = (p & 0xFFFFFFFF).to(torch.int32)
+
+    def pack_flag_bits(self, bounds, P, words, bits):
+        weights = (torch.ones(32, dtype=torch.int64) << torch.arange(32))
+        for q in range(P):
+            b, e = int(bounds[q]), int(bounds[q + 1])
+            seg = torch.zeros(words * 32, dtype=torch.int64)
+            seg[: e - b] = self.flags[b:e].to(torch.int64) != 0
+            x = (seg.view(words, 32) * weights).sum(1)
+            bits[q * words:(q + 1) * words] = (x - ((x >> 31) << 32)).to(torch.int32)   # two's complement int32
+        self.flags[:self.row_begin] = 0
+        self.flags[self.row_end:] = 0
+
+    def or_flag_bits(self, bits, P, words):
+        x = torch.zeros(words, dtype=torch.int64)
+        for q in range(P):
+            x |= bits[q * words:(q + 1) * words].to(torch.int64) & 0xFFFFFFFF
+        n = self.row_end - self.row_begin
+        unpacked = ((x.view(words, 1) >> torch.arange(32)) & 1).flatten()[:n]
+        self.flags[self.row_begin:self.row_end] = unpacked.to(torch.uint8)
+
     def sweep(self, pickless):
         C = self.labels.numpy()
         U = self.flags.numpy()
@@ -132,7 +169,9 @@ def test_two_rank_gloo_matches_emulation():
     mp.spawn(_worker, args=(world, port, out), nprocs=world, join=True)
     (C0, r0), (C1, r1) = out[0], out[1]
     assert np.array_equal(C0, C1), "replicated labels differ between ranks"
-    assert r0 == r1
+    strip = lambda r: {k: v for k, v in r.items() if k != "exchange"}   # bytes sent differ per rank
+    assert strip(r0) == strip(r1)
+    assert [x["labels"] for x in r0["exchange"]] == [x["labels"] for x in r1["exchange"]]
     g = synth.sbm(n=1500, community_size=50, avg_degree=10, mu=0.2, seed=5)
     C, changed = emulate(g, world)
     assert r0["changed"] == changed
@@ -140,3 +179,45 @@ def test_two_rank_gloo_matches_emulation():
     assert r0["converged"]
     q = oracle.modularity(oracle.CSR.from_graph(g), C0)
     assert q > 0.5
+    # the first sweep changes every label (dense all-gather), later sweeps
+    # send only the changed ones as pairs
+    modes = [x["labels"] for x in r0["exchange"]]
+    assert modes[0] == "dense" and "sparse" in modes, modes
+    assert [x["dn"] for x in r0["exchange"]] == changed
+
+
+def test_exchange_primitives_reference():
+    """The pair / bitmap encodings used by the exchange round-trip."""
+    g = synth.sbm(n=300, community_size=30, avg_degree=6, seed=2)
+    bounds = D.partition_by_edges(g.offsets, 3)
+    run = OracleShardRunner(g, *bounds[1], bounds)
+    run.reset()
+    run.snapshot()
+    b, e = bounds[1]
+    run.labels[b + 3] = 7
+    run.labels[e - 1] = 0
+    pairs = torch.full((e - b,), -5, dtype=torch.int64)
+    k = run.pack_changed(pairs)
+    assert k == 2
+    other = OracleShardRunner(g, *bounds[0], bounds)
+    other.reset()
+    other.apply_pairs(torch.cat([pairs[:k], torch.tensor([-1])]), k + 1)
+    assert int(other.labels[b + 3]) == 7 and int(other.labels[e - 1]) == 0
+    assert int((other.labels != torch.arange(g.N, dtype=torch.int32)).sum()) == 2
+    # bitmaps: rank 1's marks on every range, OR-ed into each owner
+    rng = np.random.default_rng(0)
+    fl = torch.from_numpy((rng.random(g.N) < 0.3).astype(np.uint8))
+    run.flags.copy_(fl)
+    words = (max(e_ - b_ for b_, e_ in bounds) + 31) // 32
+    bits = torch.zeros(3 * words, dtype=torch.int32)
+    bt = torch.tensor([x for x, _ in bounds] + [bounds[-1][1]])
+    run.pack_flag_bits(bt, 3, words, bits)
+    assert int(run.flags[:b].sum()) == 0 and int(run.flags[e:].sum()) == 0
+    for q in range(3):
+        own = OracleShardRunner(g, *bounds[q], bounds)
+        own.flags.zero_()
+        recv = torch.zeros(3 * words, dtype=torch.int32)
+        recv[words:2 * words] = bits[q * words:(q + 1) * words]     # from rank 1
+        own.or_flag_bits(recv, 3, words)
+        qb, qe = bounds[q]
+        assert torch.equal(own.flags[qb:qe], fl[qb:qe])

@@ -487,3 +487,57 @@ def test_distributed_driver_nccl_world1():
         assert abs(D.modularity_distributed(runner_a) - oracle.modularity(h, runner_a.labels.cpu().numpy())) < 1e-9
     finally:
         dist.destroy_process_group()
+
+
+def test_exchange_primitives_cuda_vs_reference():
+    """nulpa_pack_changed / nulpa_apply_pairs / nulpa_pack_flag_bits /
+    nulpa_or_flag_bits (the multi-GPU exchange kernels) against the
+    reference semantics of tests/test_distributed.py's CPU runner."""
+    import sys, os
+    sys.path.insert(0, os.path.dirname(__file__))
+    from test_distributed import OracleShardRunner
+    from paper_conf_ipps_sahunk25_b200 import distributed as D
+    g = GRAPHS["web"](False)
+    P = 3
+    bounds = D.partition_by_edges(g.offsets, P)
+    rng = np.random.default_rng(4)
+    for r in range(P):
+        b, e = bounds[r]
+        cu = D.CudaShardRunner(D.shard_graph(g.offsets, g.indices, None, r, P))
+        ref = OracleShardRunner(g, b, e, bounds)
+        C0 = torch.from_numpy(rng.integers(0, g.N, g.N).astype(np.int32))
+        cu.labels.copy_(C0.cuda())
+        ref.labels.copy_(C0)
+        cu.snapshot()
+        ref.snapshot()
+        C1 = C0.clone()
+        moved = torch.from_numpy(rng.random(e - b) < 0.1)
+        C1[b:e][moved] = torch.from_numpy(rng.integers(0, g.N, int(moved.sum())).astype(np.int32))
+        cu.labels.copy_(C1.cuda())
+        ref.labels.copy_(C1)
+        pc = torch.full((e - b,), -1, dtype=torch.int64, device="cuda")
+        pr = torch.full((e - b,), -1, dtype=torch.int64)
+        kc, kr = cu.pack_changed(pc), ref.pack_changed(pr)
+        assert kc == kr
+        assert torch.equal(torch.sort(pc[:kc].cpu()).values, torch.sort(pr[:kr]).values)
+        # apply onto the pre-sweep labels of another replica
+        cu.labels.copy_(C0.cuda())
+        cu.apply_pairs(torch.cat([pc[:kc], torch.full((5,), -1, dtype=torch.int64, device="cuda")]), kc + 5)
+        assert torch.equal(cu.labels.cpu()[b:e], C1[b:e]) and torch.equal(cu.labels.cpu()[:b], C0[:b])
+        # bitmaps
+        F = torch.from_numpy((rng.random(g.N) < 0.3).astype(np.uint8))
+        cu.flags.copy_(F.cuda())
+        ref.flags.copy_(F)
+        words = (max(y - x for x, y in bounds) + 31) // 32
+        bt = torch.tensor([x for x, _ in bounds] + [bounds[-1][1]], dtype=torch.int64)
+        bc = torch.zeros(P * words, dtype=torch.int32, device="cuda")
+        br = torch.zeros(P * words, dtype=torch.int32)
+        cu.pack_flag_bits(bt.cuda(), P, words, bc)
+        ref.pack_flag_bits(bt, P, words, br)
+        assert torch.equal(bc.cpu(), br)
+        assert torch.equal(cu.flags.cpu(), ref.flags)
+        recv = torch.from_numpy(rng.integers(-2**31, 2**31, P * words, dtype=np.int64).astype(np.int32))
+        cu.or_flag_bits(recv.cuda(), P, words)
+        ref.or_flag_bits(recv, P, words)
+        assert torch.equal(cu.flags.cpu(), ref.flags)
+        cu.g.close()
