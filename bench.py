@@ -42,7 +42,7 @@ BINS = ("thread", "warp", "block", "giant")
 def parse_args():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", default="web_40m_2200m")
@@ -109,9 +109,11 @@ KERNELS = {0: "k_thread", 1: "k_frontier + k_warp", 2: "k_frontier + k_warp<1024
 
 
 class Clocks:
-    """nvidia-smi sampler running during the timed region."""
+    """nvidia-smi sampler (every 20 ms) started before the timed region;
+    only the samples whose timestamps fall inside the timed region
+    (mark_start / mark_stop, wall clock) are reported."""
 
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
@@ -119,19 +121,31 @@ class Clocks:
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         self.gpu = gpu_index
         self.p = None
+        self.t0 = self.t1 = None
 
     def start(self):
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                       "--format=csv,noheader,nounits", "-lms", "20"],
                                       stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
+            return
+        for _ in range(150):                     # until the sampler writes (up to 3 s)
+            time.sleep(0.02)
+            if os.path.getsize(self.f.name) > 0:
+                break
+
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_stop(self):
+        self.t1 = time.time()
 
     def stop(self):
         if self.p is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        time.sleep(0.25)
+        time.sleep(0.1)
         self.p.terminate()
         try:
             self.p.wait(timeout=5)
@@ -140,17 +154,26 @@ class Clocks:
         self.f.flush()
         rows = [r.split(", ") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
         os.unlink(self.f.name)
-        sm = [float(r[1]) for r in rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+
+        def ts(r):
+            try:
+                import datetime
+                return datetime.datetime.strptime(r[0].strip(), "%Y/%m/%d %H:%M:%S.%f").timestamp()
+            except Exception:
+                return None
+        rows = [r for r in rows if len(r) >= 10]
+        inside = [r for r in rows if self.t0 and ts(r) is not None and self.t0 - 0.02 <= ts(r) <= (self.t1 or 1e30) + 0.02]
+        use = inside or rows
+        sm = [float(r[2]) for r in use if r[2].replace(".", "").isdigit()]
+        mx = [float(r[3]) for r in use if r[3].replace(".", "").isdigit()]
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in rows:
-            if len(r) >= 9:
-                for k, nm in enumerate(names):
-                    if r[5 + k].strip() == "Active":
-                        reasons.add(nm)
+        for r in use:
+            for k, nm in enumerate(names):
+                if r[6 + k].strip() == "Active":
+                    reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(rows)}
+                "reasons": sorted(reasons), "samples": len(use), "samples_in_timed_region": len(inside)}
 
 
 # ---------------------------------------------------------------------------
@@ -266,11 +289,13 @@ def run_ours(args):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     stats = []
     torch.cuda.synchronize()
+    clocks.mark_start()
     ev0.record(stream)
     for _ in range(args.steps):
         stats.append(gg.run(**params))
     ev1.record(stream)
     torch.cuda.synchronize()
+    clocks.mark_stop()
     ck = clocks.stop()
     ms = ev0.elapsed_time(ev1) / args.steps
     value = M / (ms / 1e3)
@@ -445,12 +470,14 @@ def run_distributed(args, rank, world, local):
     torch.cuda.synchronize()
     dist.barrier()
     st_a = runner.g.stats()
+    clocks.mark_start()
     ev0.record()
     res = None
     for _ in range(args.steps):
         res = D.lpa_distributed(runner)
     ev1.record()
     torch.cuda.synchronize()
+    clocks.mark_stop()
     dist.barrier()
     ck = clocks.stop()
     st_b = runner.g.stats()

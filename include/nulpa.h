@@ -81,18 +81,16 @@ typedef struct nulpa_params {
                                     Range [1, 1024] (distinct labels <= D <= 1023 = p1, so R5's
                                     linear continuation always finds a slot); <= block_degree
                                     sends the whole bin to the CTA kernel.  B200 default 512    */
-    int32_t first_sweep_block;   /* warp-bin schedule of the first sweep after a reset: each warp
-                                    walks blocks of this many consecutive 32-vertex record groups
-                                    (balanced block-cyclic; 1 = strided).  Larger blocks let labels
-                                    propagate along ID order within a warp as in the sequential
-                                    Algorithm 1 (better modularity) at some memory-latency cost.
-                                    Range [1, 1024]; default 192    */
-    int32_t sweep_block;         /* the same for every later sweep; default 4.  Any value > 1
-                                    hands out guided chunks of min(block, max(block / 4, groups
-                                    left / warps)) from a global counter (balance; the floor
-                                    keeps first-sweep runs >= 1536 rows at the default 192, see
-                                    DESIGN.md "Quality notes"); 1 is the static strided
-                                    schedule                                                    */
+    int32_t first_sweep_block;   /* warp-bin schedule of the first sweep after a reset.
+                                    0 (default): each warp owns one contiguous range of the
+                                    bin's 32-vertex record groups and walks it in ID order;
+                                    warps that run dry steal the far half of the most-loaded
+                                    of 32 sampled ranges (labels propagate along ID order within
+                                    a run as in the sequential Algorithm 1 -- modularity -- and
+                                    the end of the sweep is balanced; DESIGN.md "Quality
+                                    notes").  1: static strided; > 1: guided chunks of up to
+                                    this many groups from a global counter.  Range [0, 1024]   */
+    int32_t sweep_block;         /* the same for every later sweep; default 4 (guided)          */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0

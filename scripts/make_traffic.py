@@ -43,7 +43,17 @@ if binname == "warp":
     b = [dram(f) + dram(w) for f, w in zip(front, main)]
     kernels = ["k_frontier", "k_warp"]
     extra = {"k_warp_per_launch": [dram(w) for w in main], "k_frontier_per_launch": [dram(f) for f in front]}
+elif binname == "block":
+    # per sweep: the block-bin k_frontier (the one before a k_warp<..., 1024, ...>), the wide k_warp, k_block
+    wide = [k for k in ids if "k_warp" in name[k] and ", 1024" in name[k]]
+    front = [ids[ids.index(k) - 1] for k in wide]
+    blk = [next(x for x in ids[ids.index(k):] if "k_block" in name[x]) for k in wide]
+    assert all("k_frontier" in name[f] for f in front)
+    b = [dram(f) + dram(w) + dram(c) for f, w, c in zip(front, wide, blk)]
+    kernels = ["k_frontier", "k_warp<1024>", "k_block"]
+    extra = {"k_block_per_launch": [dram(c) for c in blk], "k_warp_wide_per_launch": [dram(w) for w in wide]}
 else:
+    # thread bin: every k_thread launch of a sweep (several waves on small bulk bins)
     main = [k for k in ids if "k_thread" in name[k]]
     b = [dram(k) for k in main]
     kernels = ["k_thread"]
