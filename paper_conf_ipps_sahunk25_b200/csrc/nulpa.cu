@@ -1541,9 +1541,11 @@ __global__ void __launch_bounds__(256) k_mod_degrees(const int64_t *__restrict__
 }
 
 // acc[0] += sigma_intra = sum over CSR entries (i,j) with C_i = C_j of w_ij.
-// A warp takes 32 consecutive rows (their labels / offsets in one round
-// trip) and strides over each row's entries; per-lane float64 partial sums,
-// reduced once at the end.
+// A warp takes 32 consecutive rows and streams their CSR entries as one flat,
+// coalesced range (32 entries per lane step, two steps in flight); an
+// entry's row is found by a 5-step binary search over the 33 row offsets
+// held one per lane (shuffles), its label compared with the gathered C_j.
+// Per-lane float64 partial sums, reduced once at the end.
 template <bool W>
 __global__ void __launch_bounds__(256) k_mod_intra(const int64_t *__restrict__ offsets, const int32_t *__restrict__ indices,
                                                    const float *__restrict__ weights, const int32_t *__restrict__ labels,
@@ -1553,19 +1555,42 @@ __global__ void __launch_bounds__(256) k_mod_intra(const int64_t *__restrict__ o
     const int64_t nchunks = (n_rows + 31) / 32;
     double in = 0.0;
     for (int64_t c = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); c < nchunks; c += nw) {
-        const int64_t r = c * 32 + lane;
-        int32_t cv = 0;
-        int64_t o0 = 0, o1 = 0;
-        if (r < n_rows) {
-            cv = labels[r + row_begin];
-            o0 = offsets[r];
-            o1 = offsets[r + 1];
-        }
-        for (int k = 0; k < 32; ++k) {
-            const int32_t ck = __shfl_sync(0xFFFFFFFFu, cv, k);
-            const int64_t b = __shfl_sync(0xFFFFFFFFu, o0, k), e1 = __shfl_sync(0xFFFFFFFFu, o1, k);
-            for (int64_t e = b + lane; e < e1; e += 32)
-                if (labels[ld_stream(indices + e)] == ck) in += W ? (double)ld_stream(weights + e) : 1.0;
+        const int64_t r0 = c * 32, r = r0 + lane;
+        const int64_t o_abs = offsets[min(r, n_rows)];
+        const int32_t cl = r < n_rows ? labels[r + row_begin] : 0;
+        const int64_t e0 = __shfl_sync(0xFFFFFFFFu, o_abs, 0);
+        const uint32_t ol = (uint32_t)(o_abs - e0);                   // row starts relative to the chunk
+        const uint32_t len = (uint32_t)(offsets[min(r0 + 32, n_rows)] - e0);
+        const int32_t nr = n_rows - r0 < 32 ? (int32_t)(n_rows - r0) : 32;
+        auto row_of = [&](uint32_t e) -> int32_t {                   // largest k < nr with start(k) <= e
+            int32_t k = 0;
+#pragma unroll
+            for (int st = 16; st; st >>= 1) {
+                const int32_t t = k + st;
+                const uint32_t ot = __shfl_sync(0xFFFFFFFFu, ol, t & 31);
+                if (t < nr && ot <= e) k = t;
+            }
+            return k;
+        };
+        constexpr int UM = 4;                                         // entries per lane in flight
+        for (uint32_t base = 0; base < len; base += 32 * UM) {
+            int32_t j[UM], lb[UM];
+            float w[UM];
+            bool v[UM];
+#pragma unroll
+            for (int u = 0; u < UM; ++u) {
+                const uint32_t e = base + 32 * u + lane;
+                v[u] = e < len;
+                j[u] = v[u] ? ld_stream(indices + e0 + e) : 0;
+                w[u] = W && v[u] ? ld_stream(weights + e0 + e) : 1.0f;
+            }
+#pragma unroll
+            for (int u = 0; u < UM; ++u) lb[u] = v[u] ? labels[j[u]] : 0;
+#pragma unroll
+            for (int u = 0; u < UM; ++u) {
+                const int32_t cr = __shfl_sync(0xFFFFFFFFu, cl, row_of(base + 32 * u + lane));
+                if (v[u] && lb[u] == cr) in += W ? (double)w[u] : 1.0;
+            }
         }
     }
 #pragma unroll
