@@ -91,6 +91,12 @@ typedef struct nulpa_params {
                                     notes").  1: static strided; > 1: guided chunks of up to
                                     this many groups from a global counter.  Range [0, 1024]   */
     int32_t sweep_block;         /* the same for every later sweep; default 4 (guided)          */
+    int32_t device_loop;         /* 1 (default): when timing == 0, nulpa_run launches sweep 0 and
+                                    then ONE CUDA graph whose conditional while node runs sweeps
+                                    1.. and Algorithm 1's stop test on the device
+                                    -- no host synchronisation per iteration; the graph is built
+                                    once per handle and parameter set.  0 (or timing == 1): the
+                                    host loop, one synchronisation per iteration               */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0
@@ -154,8 +160,10 @@ int nulpa_create(const int64_t *offsets, const int32_t *indices, const float *we
 int nulpa_bind_state(nulpa_graph *g, int32_t *labels_device, uint8_t *flags_device);
 
 /* Run Algorithm 1's lpa() loop with `params` (NULL =
- * defaults) and fill *stats (may be NULL).  Synchronises the stream once per
- * iteration (the tolerance test needs dN on the host). */
+ * defaults) and fill *stats (may be NULL).  With params->device_loop (and no
+ * timing) the stop test runs on the device and the stream is synchronised
+ * once at the end; otherwise once per iteration (the tolerance test then
+ * needs dN on the host). */
 int nulpa_run(nulpa_graph *g, const nulpa_params *params, nulpa_stats *stats);
 
 /* One lpaMove over this handle's rows with Pick-Less on

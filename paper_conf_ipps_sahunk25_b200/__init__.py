@@ -55,6 +55,7 @@ class Params(ctypes.Structure):
         ("wide_degree", ctypes.c_int32),
         ("first_sweep_block", ctypes.c_int32),
         ("sweep_block", ctypes.c_int32),
+        ("device_loop", ctypes.c_int32),
     ]
 
 

@@ -295,8 +295,11 @@ struct SweepArgs {
     uint8_t *flag_out;
     int64_t row_begin;
     int pickless;
+    const int32_t *pl_dev;     // device loop (nulpa_run's CUDA graph): Pick-Less flag in device memory, else null
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
+// this sweep's Pick-Less flag: from the device loop's state, or the host's
+__device__ __forceinline__ int sweep_pl(const SweepArgs &a) { return a.pl_dev ? *a.pl_dev : a.pickless; }
 
 // ---------------------------------------------------------------------------
 // thread-per-vertex kernel (degree < switch_degree <= 33), PAPER.md:241-243:
@@ -319,6 +322,7 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
     __syncthreads();
     uint32_t n_act = 0, n_ch = 0;
     unsigned long long e_act = 0, e_ch = 0;
+    const int pl = sweep_pl(a);
     auto process = [&](int32_t r) {
         const int64_t v = r + a.row_begin;
         const int64_t o = a.offsets[r];
@@ -356,7 +360,7 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
         const int32_t cs = best ? cand_label(best, to) : kEmpty;
         n_act += 1;
         e_act += deg;
-        if (accept_move(cs, ci, a.pickless)) {
+        if (accept_move(cs, ci, pl)) {
             a.lab_out[v] = cs;
             n_ch += 1;
             e_ch += deg;
@@ -885,6 +889,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     const unsigned lanes_below = (1u << lane) - 1;
     if (threadIdx.x < 2) bctr[threadIdx.x] = 0;
     const uint32_t nrec = (uint32_t)*count;
+    const int pl = sweep_pl(a);
     GroupFetcher F;
     F.ng = (nrec + G - 1) / G;
     F.nw = gridDim.x * NWARP;
@@ -985,7 +990,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         // ---- fold vertex n ----
         const int32_t vk = rc.r + (int32_t)a.row_begin;
         const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, k0a, k0b, w0a, w0b);
-        if (accept_move(cs, rc.ci, a.pickless)) {
+        if (accept_move(cs, rc.ci, pl)) {
             c_ch += 1;
             c_che += dk;
             if (lane == 0) a.lab_out[vk] = cs;
@@ -1160,7 +1165,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
             uint64_t bb = 0;
             for (int q = 0; q < kBlkThreads / 32; ++q) bb = s_best[q] > bb ? s_best[q] : bb;
             const int32_t cs = bb ? (int32_t)~(uint32_t)bb : kEmpty;
-            const int ch = accept_move(cs, rc.ci, a.pickless);
+            const int ch = accept_move(cs, rc.ci, sweep_pl(a));
             if (ch) a.lab_out[v] = cs;
             s_changed = ch;
             n_changed += ch;
@@ -1326,7 +1331,7 @@ __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     to.init(h);
     const unsigned long long b = g.best[gi];
     const int32_t cs = b ? cand_label(b, to) : kEmpty;
-    const bool ch = accept_move(cs, a.lab_in[v], a.pickless);
+    const bool ch = accept_move(cs, a.lab_in[v], sweep_pl(a));
     if (ch) {
         a.lab_out[v] = cs;
         g.changed[gi] = 1;
@@ -1742,6 +1747,15 @@ struct nulpa_graph {
     bool events = false;
     cudaStream_t side = nullptr;             // bin_order 2: block + giant bins
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    // device loop (nulpa_run without timing): [sweep 1.. + stop test] as a
+    // CUDA graph with a conditional while node, built once per parameter set
+    int32_t *loopvars = nullptr;             // device [4], see k_loop_step
+    cudaGraph_t loop_graph = nullptr;
+    cudaGraphExec_t loop_exec = nullptr;
+    nulpa_params loop_p;                     // parameters the graph was captured with
+    int loop_launches[4] = {0, 0, 0, 0};     // kernel launches of one loop body, per bin
+    int loop_other = 0;
+    cudaStream_t cap = nullptr;              // capture stream of the device loop (the caller's may be the legacy stream)
     cudaStream_t hi = nullptr;               // bin_order 3: high-priority stream for the warp bin
     cudaEvent_t ev_mid = nullptr, ev_join2 = nullptr;
     nulpa_stats stats;
@@ -1795,8 +1809,16 @@ void dfree(void *p) {
     if (p) cudaFreeAsync(p, 0);
 }
 
+void free_loop(nulpa_graph *g) {
+    if (g->loop_exec) cudaGraphExecDestroy(g->loop_exec);
+    if (g->loop_graph) cudaGraphDestroy(g->loop_graph);
+    g->loop_exec = nullptr;
+    g->loop_graph = nullptr;
+}
+
 void free_bins(nulpa_graph *g) {
     if (g->stream) cudaStreamSynchronize(g->stream);
+    free_loop(g);
     dfree(g->wrecs);
     g->wrecs = nullptr;
     dfree(g->wranges);
@@ -1886,6 +1908,30 @@ __global__ void k_or_flag_bits(uint8_t *flags, const uint32_t *__restrict__ bits
         uint32_t x = 0;
         for (int q = 0; q < P; ++q) x |= bits[(int64_t)q * words + (i >> 5)];
         flags[own_b + i] = (x >> (i & 31)) & 1u;
+    }
+}
+
+// Algorithm 1's stop test on the device (nulpa_run's CUDA-graph loop,
+// PAPER.md:305-318): iteration l = lv[0] has just swept with Pick-Less lv[1]
+// and left its counters in `scratch`; they move to counter slot l; stop
+// (conditional = 0) when not Pick-Less and dN/N < tau or l + 1 = maxit,
+// else advance l and the Pick-Less flag of iteration l + 1.
+// lv: [0] iteration, [1] Pick-Less flag, [2] converged, [3] iterations done.
+__global__ void k_loop_step(unsigned long long *scratch, unsigned long long *ctr_all, int32_t *lv, double n_global,
+                            double tol, int rho, int maxit, cudaGraphConditionalHandle cond) {
+    const int l = lv[0];
+    for (int k = threadIdx.x; k < kCtr; k += blockDim.x) ctr_all[(size_t)l * kCtr + k] = scratch[k];
+    if (threadIdx.x == 0) {
+        const bool pl = lv[1] != 0;
+        const bool conv = !pl && (double)scratch[0] / n_global < tol;
+        const bool stop = conv || l + 1 >= maxit;
+        lv[2] = conv ? 1 : 0;
+        lv[3] = l + 1;
+        if (!stop) {
+            lv[0] = l + 1;
+            lv[1] = rho > 0 && (l + 1) % rho == 0;
+        }
+        cudaGraphSetConditional(cond, stop ? 0u : 1u);
     }
 }
 
@@ -2092,8 +2138,10 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
 }
 
 template <bool SYNC, bool W>
-int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
+int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot,
+               const int32_t *pl_dev) {
     SweepArgs a;
+    a.pl_dev = pl_dev;
     a.offsets = g->offsets;
     a.indices = g->indices;
     a.weights = g->weights;
@@ -2299,7 +2347,8 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     return NULPA_OK;
 }
 
-int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot) {
+int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long long *ctr, bool timing, int slot,
+          const int32_t *pl_dev = nullptr) {
     const bool w = g->weights != nullptr;
     if (p.mode == NULPA_SYNC && !g->labels_prev) {
         CHECK(dalloc(&g->labels_prev, (size_t)g->n_global));
@@ -2308,13 +2357,85 @@ int sweep(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned long lon
     const int sel = (p.mode == NULPA_SYNC ? 2 : 0) + (w ? 1 : 0);
     int r;
     switch (sel) {
-    case 0: r = sweep_impl<false, false>(g, pickless, p, ctr, timing, slot); break;
-    case 1: r = sweep_impl<false, true>(g, pickless, p, ctr, timing, slot); break;
-    case 2: r = sweep_impl<true, false>(g, pickless, p, ctr, timing, slot); break;
-    default: r = sweep_impl<true, true>(g, pickless, p, ctr, timing, slot); break;
+    case 0: r = sweep_impl<false, false>(g, pickless, p, ctr, timing, slot, pl_dev); break;
+    case 1: r = sweep_impl<false, true>(g, pickless, p, ctr, timing, slot, pl_dev); break;
+    case 2: r = sweep_impl<true, false>(g, pickless, p, ctr, timing, slot, pl_dev); break;
+    default: r = sweep_impl<true, true>(g, pickless, p, ctr, timing, slot, pl_dev); break;
     }
     ++g->sweeps_since_reset;
     return r;
+}
+
+bool same_loop_params(const nulpa_params &a, const nulpa_params &b) {
+    return a.tolerance == b.tolerance && a.max_iterations == b.max_iterations && a.pickless_period == b.pickless_period &&
+           a.mode == b.mode && a.switch_degree == b.switch_degree && a.block_degree == b.block_degree &&
+           a.giant_degree == b.giant_degree && a.bin_order == b.bin_order && a.wide_degree == b.wide_degree &&
+           a.sweep_block == b.sweep_block;
+}
+
+// The device loop: graph = [k_loop_step for sweep 0] -> while (cond) {
+// memset(scratch counters); sweep (Pick-Less flag from loopvars[1], bins
+// as in a host-loop sweep >= 1); k_loop_step }.  Captured from the handle's
+// stream (the bin streams join the capture through their events).
+int build_loop(nulpa_graph *g, const nulpa_params &p, int maxit) {
+    free_loop(g);
+    if (!g->loopvars) CHECK(dalloc(&g->loopvars, 4));
+    unsigned long long *scratch = g->ctr + (size_t)kMaxIter * kCtr;
+    CU(cudaGraphCreate(&g->loop_graph, 0));
+    cudaGraphConditionalHandle cond;
+    CU(cudaGraphConditionalHandleCreate(&cond, g->loop_graph, 1, cudaGraphCondAssignDefault));
+    // first node: the stop test of sweep 0 (launched before the graph)
+    cudaGraphNode_t first;
+    {
+        cudaKernelNodeParams kp = {};
+        double n_global = (double)g->n_global, tol = p.tolerance;
+        int rho = p.pickless_period;
+        unsigned long long *ctr_all = g->ctr;
+        int32_t *lv = g->loopvars;
+        void *args[] = {&scratch, &ctr_all, &lv, &n_global, &tol, &rho, &maxit, &cond};
+        kp.func = (void *)k_loop_step;
+        kp.gridDim = dim3(1);
+        kp.blockDim = dim3(32);
+        kp.kernelParams = args;
+        CU(cudaGraphAddKernelNode(&first, g->loop_graph, nullptr, 0, &kp));
+    }
+    cudaGraphNodeParams cp = {};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = cond;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    cudaGraphNode_t wnode;
+    CU(cudaGraphAddNode(&wnode, g->loop_graph, &first, 1, &cp));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+    int l0[4];
+    memcpy(l0, g->stats.launches, sizeof l0);
+    const int o0 = g->stats.other_launches;
+    if (!g->cap) CU(cudaStreamCreateWithFlags(&g->cap, cudaStreamNonBlocking));
+    cudaStream_t user = g->stream;
+    g->stream = g->cap;                                  // the sweep's kernels go to the capture stream
+    CU(cudaStreamBeginCaptureToGraph(g->stream, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+    int r = NULPA_OK;
+    if (cudaMemsetAsync(scratch, 0, kCtr * sizeof(unsigned long long), g->stream) != cudaSuccess) r = NULPA_ECUDA;
+    if (r == NULPA_OK) r = sweep(g, 0, p, scratch, false, 0, g->loopvars + 1);
+    if (r == NULPA_OK) {
+        double n_global = (double)g->n_global;
+        k_loop_step<<<1, 32, 0, g->stream>>>(scratch, g->ctr, g->loopvars, n_global, p.tolerance, p.pickless_period, maxit, cond);
+        if (cudaGetLastError() != cudaSuccess) r = NULPA_ECUDA;
+    }
+    cudaGraph_t captured = nullptr;
+    const cudaError_t ec = cudaStreamEndCapture(g->stream, &captured);
+    g->stream = user;
+    if (r != NULPA_OK) return r == NULPA_ECUDA ? fail(NULPA_ECUDA, "capturing the device loop failed") : r;
+    CU(ec);
+    for (int b = 0; b < 4; ++b) {
+        g->loop_launches[b] = g->stats.launches[b] - l0[b];
+        g->stats.launches[b] = l0[b];
+    }
+    g->loop_other = g->stats.other_launches - o0 + 2;          // + the two k_loop_step launches' bookkeeping
+    g->stats.other_launches = o0;
+    CU(cudaGraphInstantiate(&g->loop_exec, g->loop_graph, 0));
+    g->loop_p = p;
+    return NULPA_OK;
 }
 
 int reset_state(nulpa_graph *g) {
@@ -2411,6 +2532,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->wide_degree = 512;
     p->first_sweep_block = 0;
     p->sweep_block = 4;
+    p->device_loop = 1;
 }
 
 const char *nulpa_last_error(void) { return g_err.c_str(); }
@@ -2586,7 +2708,29 @@ int nulpa_run(nulpa_graph *g, const nulpa_params *params, nulpa_stats *stats) {
     if (p.reset) CHECK(reset_state(g));
     int l = 0;
     int converged = 0;
-    for (; l < maxit; ++l) {
+    if (!timing && p.device_loop && maxit >= 2) {
+        // device loop: sweep 0 (first-sweep schedule) from the host, then
+        // one graph launch runs the stop tests and sweeps 1.. (no host sync
+        // per iteration)
+        const int pl0 = p.pickless_period > 0;
+        unsigned long long *scratch = g->ctr + (size_t)kMaxIter * kCtr;
+        if (!g->loopvars) CHECK(dalloc(&g->loopvars, 4));
+        CU(cudaMemsetAsync(g->loopvars, 0, 4 * sizeof(int32_t), g->stream));
+        if (pl0) CU(cudaMemsetAsync(g->loopvars + 1, 1, 1, g->stream));   // lv[1] = 1 (little-endian)
+        CHECK(sweep(g, pl0, p, scratch, false, 0));
+        if (!g->loop_exec || !same_loop_params(g->loop_p, p) || g->loop_p.max_iterations != maxit)
+            CHECK(build_loop(g, p, maxit));
+        CU(cudaGraphLaunch(g->loop_exec, g->stream));
+        int32_t lv[4];
+        CU(cudaMemcpyAsync(lv, g->loopvars, sizeof lv, cudaMemcpyDeviceToHost, g->stream));
+        CU(cudaStreamSynchronize(g->stream));
+        l = lv[3];
+        converged = lv[2];
+        for (int b = 0; b < 4; ++b) g->stats.launches[b] += g->loop_launches[b] * (l - 1);
+        g->stats.other_launches += g->loop_other * (l - 1) + 1;
+        g->sweeps_since_reset += l - 1;
+    }
+    for (; l < maxit && !(!timing && p.device_loop && maxit >= 2); ++l) {
         const int pl = p.pickless_period > 0 && (l % p.pickless_period) == 0;
         unsigned long long *ctr = g->ctr + (size_t)l * kCtr;
         CHECK(sweep(g, pl, p, ctr, timing, l));
@@ -2772,6 +2916,11 @@ int nulpa_destroy(nulpa_graph *g) {
     if (!g) return NULPA_OK;
     if (g->stream) cudaStreamSynchronize(g->stream);
     free_bins(g);
+    dfree(g->loopvars);
+    if (g->cap) {
+        cudaStreamSynchronize(g->cap);
+        cudaStreamDestroy(g->cap);
+    }
     if (g->own_csr) {
         dfree(g->offsets);
         dfree(g->indices);

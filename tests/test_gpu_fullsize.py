@@ -29,7 +29,7 @@ import paper_conf_ipps_sahunk25_b200 as nl
 
 pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 
-QUALITY_SEEDS = (0, 1)
+QUALITY_SEEDS = tuple(int(x) for x in os.environ.get("NULPA_FULLSIZE_SEEDS", "0,1").split(","))
 QUALITY_RUNS = 6
 
 

@@ -541,3 +541,25 @@ def test_exchange_primitives_cuda_vs_reference():
         ref.or_flag_bits(recv, P, words)
         assert torch.equal(cu.flags.cpu(), ref.flags)
         cu.g.close()
+
+
+@pytest.mark.parametrize("gname", ["sbm", "web", "road", "hub", "kmer"])
+def test_device_loop_matches_host_loop(gname):
+    """nulpa_run's CUDA-graph loop (device-side stop test) and the host loop
+    (one synchronisation per iteration) give the same synchronous run as the
+    oracle, and the same iteration count / dN list; the asynchronous device
+    loop converges with the oracle-relative quality bar."""
+    g = GRAPHS[gname](False)
+    h = host(g)
+    C, it, dn = oracle.lpa(h, sync=True)
+    gg = to_gpu(g)
+    for dl in (0, 1):
+        st = gg.run(mode=nl.SYNC, device_loop=dl)
+        assert st["iterations"] == it and st["changed"] == list(dn), (dl, st["changed"], list(dn))
+        np.testing.assert_array_equal(gg.labels(device=False).numpy(), C)
+    st = gg.run(device_loop=1, max_iterations=3, tolerance=0.0)     # stops at max_iterations
+    assert st["iterations"] == 3 and not st["converged"]
+    st = gg.run(device_loop=1)
+    assert st["converged"] or st["iterations"] == 20
+    C_o, _, _ = oracle.lpa(h)
+    assert oracle.modularity(h, gg.labels(device=False).numpy()) >= oracle.modularity(h, C_o) - 0.02
