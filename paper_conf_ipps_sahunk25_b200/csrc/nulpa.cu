@@ -675,6 +675,9 @@ constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
 #ifndef NULPA_WIDE_GROUP
 #define NULPA_WIDE_GROUP 4
 #endif
+#ifndef NULPA_WIDE_TMA
+#define NULPA_WIDE_TMA 1                 // block bin below wide_degree: TMA k_block (128 threads) instead of the wide k_warp
+#endif
 #ifndef NULPA_WIDE_K
 #define NULPA_WIDE_K 2                   // wide schedule: guided chunks of <= this many groups
 #endif
@@ -1057,11 +1060,11 @@ __device__ __forceinline__ void tma_load_1d(uint32_t dst, const void *src, uint3
                  ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
 }
 
-// R: label gathers per thread (rows of up to R * kBlkThreads entries);
+// NT threads per CTA (one vertex); R: label gathers per thread (rows of up to R * NT entries);
 // rowcap: entries per row buffer (>= max degree + 4, multiple of 4);
 // cap: table slots (>= p1 of the largest degree).
-template <bool SYNC, bool W, int R>
-__global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *__restrict__ recs,
+template <bool SYNC, bool W, int R, int NT>
+__global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restrict__ recs,
                                                         const unsigned long long *__restrict__ count, int cap,
                                                         int rowcap) {
     extern __shared__ __align__(16) uint8_t dyn_b[];
@@ -1071,7 +1074,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
     int32_t *rowi = reinterpret_cast<int32_t *>(Hf + cap);            // 2 index buffers of rowcap
     float *roww = reinterpret_cast<float *>(rowi + 2 * rowcap);       // 2 weight buffers (W)
     __shared__ __align__(8) uint64_t s_bar[2];
-    __shared__ uint64_t s_best[kBlkThreads / 32];
+    __shared__ uint64_t s_best[NT / 32];
     __shared__ int s_changed;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(&s_bar[0]);
@@ -1108,7 +1111,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         const int64_t v = rc.r + a.row_begin;
         Hash h;
         h.init(deg);
-        for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {   // hashtableClear
+        for (uint32_t q = threadIdx.x; q < h.p1; q += NT) {   // hashtableClear
             Hk[q] = kEmpty;
             Hc[q] = 0;
             Hf[q] = 0.0f;
@@ -1121,7 +1124,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         float w[R];
 #pragma unroll
         for (int u = 0; u < R; ++u) {
-            const uint32_t e = (uint32_t)(u * kBlkThreads) + threadIdx.x;
+            const uint32_t e = (uint32_t)(u * NT) + threadIdx.x;
             key[u] = kEmpty;
             w[u] = 1.0f;
             if (e < deg) {
@@ -1133,7 +1136,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         __syncthreads();                                             // table cleared
 #pragma unroll
         for (int u = 0; u < R; ++u) {
-            if ((uint32_t)(u * kBlkThreads) + (uint32_t)(wid * 32) >= deg) break;   // warp-uniform
+            if ((uint32_t)(u * NT) + (uint32_t)(wid * 32) >= deg) break;   // warp-uniform
             const unsigned grp = __match_any_sync(0xFFFFFFFFu, key[u]);
             const bool leader = key[u] != kEmpty && (grp & ((1u << lane) - 1)) == 0;
             const bool eq = !W || __all_sync(0xFFFFFFFFu, key[u] == kEmpty || w[u] == 1.0f);
@@ -1151,7 +1154,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         __syncthreads();                                             // table complete
         // hashtableMaxKey: (total, smallest label) as one 64-bit max
         uint64_t best = 0;
-        for (uint32_t q = threadIdx.x; q < h.p1; q += kBlkThreads) {
+        for (uint32_t q = threadIdx.x; q < h.p1; q += NT) {
             const int32_t kk = Hk[q];
             if (kk == kEmpty) continue;
             const float t = __fadd_rn((float)Hc[q], Hf[q]);
@@ -1163,7 +1166,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         __syncthreads();
         if (threadIdx.x == 0) {
             uint64_t bb = 0;
-            for (int q = 0; q < kBlkThreads / 32; ++q) bb = s_best[q] > bb ? s_best[q] : bb;
+            for (int q = 0; q < NT / 32; ++q) bb = s_best[q] > bb ? s_best[q] : bb;
             const int32_t cs = bb ? (int32_t)~(uint32_t)bb : kEmpty;
             const int ch = accept_move(cs, rc.ci, sweep_pl(a));
             if (ch) a.lab_out[v] = cs;
@@ -1173,7 +1176,7 @@ __global__ void __launch_bounds__(kBlkThreads) k_block(SweepArgs a, const VRec *
         }
         __syncthreads();
         if (s_changed)
-            for (uint32_t e = threadIdx.x; e < deg; e += kBlkThreads) a.flag_out[ri[e]] = 1;
+            for (uint32_t e = threadIdx.x; e < deg; e += NT) a.flag_out[ri[e]] = 1;
         __syncthreads();                                             // row buffer b and s_changed reusable
     }
     if (threadIdx.x == 0 && n_changed) {
@@ -2206,10 +2209,31 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             // frontier split at wide_degree: warp-per-vertex (1023-slot tables) below, CTA-per-vertex above
             if (!g->brecs) CHECK(dalloc(reinterpret_cast<VRec **>(&g->brecs), (size_t)(2 * n)));
             VRec *rw = reinterpret_cast<VRec *>(g->brecs), *rb = rw + n;
+            // k_block: table of the largest p1, two TMA row buffers
+            auto launch_block = [&](auto kern, int nt, int maxdeg, const VRec *recs_b, unsigned long long *cnt) -> int {
+                const int cap = (int)capacity_p1((uint32_t)maxdeg) + 1;
+                const int rowcap = (maxdeg + 4 + 3) & ~3;
+                const size_t smem = (size_t)cap * 12 + (size_t)rowcap * 4 * 2 * (W ? 2 : 1);
+                CU(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                int per_sm = 0;
+                CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, nt, smem));
+                kern<<<grid_for(n, 1, sms * std::max(1, per_sm)), nt, smem, cs>>>(a, recs_b, cnt, cap, rowcap);
+                CU(cudaGetLastError());
+                return NULPA_OK;
+            };
             const uint32_t split = (uint32_t)std::max(p.wide_degree, p.block_degree);
             k_frontier<SYNC><<<grid_for(n, kFrontTile, sms * 8), kFrontThreads, 0, cs>>>(a, g->bin_list[2], n, 2, rw, ctr + kCtrRecsW,
                                                                           split, rb, ctr + kCtrRecsB);
-            if (split > (uint32_t)p.block_degree) {
+            if (split > (uint32_t)p.block_degree && NULPA_WIDE_TMA) {
+                // degree < split (<= 1023): k_block with 4 warps per vertex, 1023-slot
+                // tables and 1 KB row buffers -- many vertices in flight per SM
+                const int md = (int)split - 1;
+                if (md + 3 <= 4 * 128)
+                    CHECK(launch_block(k_block<SYNC, W, 4, 128>, 128, md, rw, ctr + kCtrRecsW));
+                else
+                    CHECK(launch_block(k_block<SYNC, W, 8, 128>, 128, md, rw, ctr + kCtrRecsW));
+                g->stats.launches[2] += 1;
+            } else if (split > (uint32_t)p.block_degree) {
                 const WarpSched ws{SCHED_GUIDED, NULPA_WIDE_K, ctr + kCtrSchedB, nullptr};
                 if (o32)
                     k_warp<SYNC, W, kWideSlots, true><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
@@ -2217,21 +2241,9 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                     k_warp<SYNC, W, kWideSlots, false><<<sms * kWideCtasPerSm, kWideWarps * 32, 0, cs>>>(a, rw, ctr + kCtrRecsW, 2, ws);
                 g->stats.launches[2] += 1;
             }
-            // k_block: table of the largest p1, two TMA row buffers
             const int maxdeg = std::max(1, p.giant_degree - 1);
-            const int cap = (int)capacity_p1((uint32_t)maxdeg) + 1;
-            const int rowcap = (maxdeg + 4 + 3) & ~3;
-            const size_t smem = (size_t)cap * 12 + (size_t)rowcap * 4 * 2 * (W ? 2 : 1);
-            auto launch_block = [&](auto kern) -> int {
-                CU(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-                int per_sm = 0;
-                CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBlkThreads, smem));
-                kern<<<grid_for(n, 1, sms * std::max(1, per_sm)), kBlkThreads, smem, cs>>>(a, rb, ctr + kCtrRecsB, cap, rowcap);
-                CU(cudaGetLastError());
-                return NULPA_OK;
-            };
-            if (maxdeg + 3 <= 8 * kBlkThreads) CHECK(launch_block(k_block<SYNC, W, 8>));
-            else CHECK(launch_block(k_block<SYNC, W, 16>));
+            if (maxdeg + 3 <= 8 * kBlkThreads) CHECK(launch_block(k_block<SYNC, W, 8, kBlkThreads>, kBlkThreads, maxdeg, rb, ctr + kCtrRecsB));
+            else CHECK(launch_block(k_block<SYNC, W, 16, kBlkThreads>, kBlkThreads, maxdeg, rb, ctr + kCtrRecsB));
             g->stats.launches[2] += 2;
         }
         CHECK(rec(2, 1));
