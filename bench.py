@@ -523,8 +523,11 @@ def run_distributed(args, rank, world, local):
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                 "config": {"workload": args.config, "N": shard.N_global, "M": shard.M_global, "weights": args.weights,
-                           "parallelism": f"vertex range split by edge count over {world} GPUs; per sweep NCCL all-gather of labels, reduce-scatter(MAX) of flags"},
+                           "parallelism": f"vertex range split by edge count over {world} GPUs; per sweep: changed labels "
+                                          "as (vertex, label) pairs over an NCCL all-gather (dense all-gather of the label "
+                                          "ranges when > N/8 changed), marks as per-rank bitmaps over an all-to-all"},
                 "iterations": res["iterations"], "changed": res["changed"], "modularity": q,
+                "exchange_last_run": res.get("exchange"),
                 "gpu_launches": launches, "clocks": ck}
         if e2e_line:
             line["e2e"] = e2e_line

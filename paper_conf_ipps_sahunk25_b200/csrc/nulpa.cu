@@ -296,6 +296,7 @@ struct SweepArgs {
     int64_t row_begin;
     int pickless;
     const int32_t *pl_dev;     // device loop (nulpa_run's CUDA graph): Pick-Less flag in device memory, else null
+    int first;                 // first sweep after a reset (labels mostly distinct)
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 // this sweep's Pick-Less flag: from the device loop's state, or the host's
@@ -675,6 +676,12 @@ constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
 #ifndef NULPA_WIDE_GROUP
 #define NULPA_WIDE_GROUP 4
 #endif
+#ifndef NULPA_T255_MAX
+#define NULPA_T255_MAX 64                // k_warp: 255-slot tables below this degree, 511 above
+#endif
+#ifndef NULPA_FIRST_BIG
+#define NULPA_FIRST_BIG 0                // 1: 511-slot tables for every degree in the first sweep
+#endif
 #ifndef NULPA_WIDE_TMA
 #define NULPA_WIDE_TMA 1                 // block bin below wide_degree: TMA k_block (128 threads) instead of the wide k_warp
 #endif
@@ -860,7 +867,7 @@ __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, i
         if constexpr (SLOTS == kWideSlots) {
             table_row(std::integral_constant<uint32_t, kWideSlots - 1>());
         } else {
-            if (dk < 64) table_row(std::integral_constant<uint32_t, 255>());
+            if (dk < NULPA_T255_MAX && !(NULPA_FIRST_BIG && a.first)) table_row(std::integral_constant<uint32_t, 255>());
             else table_row(std::integral_constant<uint32_t, 511>());
         }
     }
@@ -2145,6 +2152,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
                const int32_t *pl_dev) {
     SweepArgs a;
     a.pl_dev = pl_dev;
+    a.first = g->sweeps_since_reset == 0;
     a.offsets = g->offsets;
     a.indices = g->indices;
     a.weights = g->weights;

@@ -88,9 +88,16 @@ def test_social_and_road_sync_sweep_whole_vector(config):
     h = host_csr(g)
     for C0, U0, pl in states(g.N, 6):
         sync_sweep_whole(g, h, None, C0, U0, pl)
-    gg = nl.Graph(g.offsets, g.indices)
+    # the production run at full size: converges, modularity >= the
+    # asynchronous oracle's - 0.02 (bench configuration: stored weights = ones)
+    ones = torch.ones(g.M, dtype=torch.float32, device="cuda")
+    gg = nl.Graph(g.offsets, g.indices, ones)
     st = gg.run()
     assert st["converged"] or st["iterations"] == 20
+    C_o, _, _ = oracle.lpa(h)
+    q_o = oracle.modularity(h, C_o)
+    q_g = gg.modularity()
+    assert q_g >= q_o - 0.02, (config, q_g, q_o)
     gg.close()
 
 
