@@ -234,11 +234,15 @@ __device__ __forceinline__ float group_sum(unsigned grp, float x, unsigned maxn)
     return x;
 }
 
-// k_warp tables store the tag k + 1 for label k (labels are >= 0 and < 2^31 - 1),
-// so an empty slot (tag 0, value 0.0f) is all-zero and hashtableClear is a
-// 16-byte store of the zero register (no per-vertex register set-up).
-constexpr uint32_t kTagEmpty = 0u;
-__device__ __forceinline__ uint32_t kv_tag(int32_t k) { return (uint32_t)k + 1u; }
+// k_warp tables store for label k the tag (k + 1) | (epoch << kbits), where
+// kbits = bit length of the number of labels and the epoch counts the
+// vertices a warp has folded since its table was last zeroed (1 ..
+// 2^(32-kbits) - 1).  A slot whose tag is below epoch << kbits -- zeroed, or
+// written for an earlier vertex -- is empty for the current vertex, so
+// hashtableClear is a counter increment, and the table is
+// zeroed (16-byte stores of the zero register) only when the epoch wraps:
+// every 63 vertices at N = 40M (kbits 26); every vertex when N >= 2^30.
+__device__ __forceinline__ uint32_t kv_tag(int32_t k, uint32_t epb) { return (uint32_t)k + 1u + epb; }
 __device__ __forceinline__ void sts_v4_empty(uint32_t addr) {
     asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(addr), "r"(0u) : "memory");
 }
@@ -269,12 +273,49 @@ __device__ __forceinline__ bool accept_move(int32_t cstar, int32_t ci, int pickl
 #ifndef NULPA_STREAM_LOAD
 #define NULPA_STREAM_LOAD 2              // 0: ld.global.cs (evict-first); 1: ld.global.nc; 2: plain ld.global
 #endif
+#ifndef NULPA_GATHER_POLICY
+#define NULPA_GATHER_POLICY 0            // label gathers C[j]: 0 plain; 1 L2 evict_last (fraction 1); 2 evict_last (fraction 0.5)
+#endif
+// 32-bit loads with an L2 cache-policy hint (createpolicy + ld.global.L2::cache_hint)
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_last(float f) {
+    uint64_t p;
+    if (f >= 1.0f) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    else asm("createpolicy.fractional.L2::evict_last.b64 %0, 0.5;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ int32_t ld_hint(const int32_t *p, uint64_t pol) {
+    int32_t v;
+    asm volatile("ld.global.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ float ld_hint(const float *p, uint64_t pol) {
+    float v;
+    asm volatile("ld.global.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+}
 template <typename T>
 __device__ __forceinline__ T ld_stream(const T *p) {
 #if NULPA_STREAM_LOAD == 0
     return __ldcs(p);
 #elif NULPA_STREAM_LOAD == 1
     return __ldg(p);
+#elif NULPA_STREAM_LOAD == 3
+    return ld_hint(p, l2_policy_evict_first());
+#else
+    return *p;
+#endif
+}
+// a label gather C[j]
+__device__ __forceinline__ int32_t ld_label(const int32_t *p) {
+#if NULPA_GATHER_POLICY == 1
+    return ld_hint(p, l2_policy_evict_last(1.0f));
+#elif NULPA_GATHER_POLICY == 2
+    return ld_hint(p, l2_policy_evict_last(0.5f));
 #else
     return *p;
 #endif
@@ -297,6 +338,7 @@ struct SweepArgs {
     int pickless;
     const int32_t *pl_dev;     // device loop (nulpa_run's CUDA graph): Pick-Less flag in device memory, else null
     int first;                 // first sweep after a reset (labels mostly distinct)
+    uint32_t kbits;            // bit length of the number of labels (k_warp table tags)
     unsigned long long *ctr;   // kCtr counters of this iteration
 };
 // this sweep's Pick-Less flag: from the device loop's state, or the host's
@@ -445,7 +487,27 @@ constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 // The value update is old value + x (an empty slot holds 0.0f), stored by
 // the lane that owns the label's slot.  `need` lanes probe; on return they
 // are done (need = false) or collided.
-__device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, float x, bool &need, float &V) {
+// Every lane reads (lanes that do not probe read the slot of their own
+// group's key -- the leader's address -- or of kEmpty, so the read is a
+// broadcast and costs no extra wavefront; no default values to set up).
+// NULPA_WARP_SYNC 0 drops the bar.warp.sync between the claim store and the
+// re-read: the warp is converged here (every caller is warp-synchronous
+// code with full-mask votes) and its shared-memory instructions complete in
+// order, and every re-reading lane stored to that address itself.
+#ifndef NULPA_WARP_SYNC
+#define NULPA_WARP_SYNC 1
+#endif
+#ifndef NULPA_EPOCH
+#define NULPA_EPOCH 1                    // 0: zero the k_warp table before every vertex
+#endif
+#if NULPA_WARP_SYNC
+#define KV_WSYNC "bar.warp.sync 0xFFFFFFFF;\n\t"
+__device__ __forceinline__ void wsync() { __syncwarp(); }
+#else
+#define KV_WSYNC ""
+__device__ __forceinline__ void wsync() { asm volatile("" ::: "memory"); }
+#endif
+__device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, uint32_t epb, float x, bool &need, float &V) {
     uint32_t n = need, vb = __float_as_uint(V);
     asm volatile(
         "{\n\t"
@@ -453,16 +515,14 @@ __device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, float x, bo
         ".reg .b32 ck, now;\n\t"
         ".reg .f32 cv, nv;\n\t"
         "setp.ne.b32 pn, %0, 0;\n\t"
-        "mov.b32 ck, 0xFFFFFFFF;\n\t"
-        "mov.f32 cv, 0f00000000;\n\t"
-        "@pn ld.shared.v2.b32 {ck, cv}, [%2];\n\t"
-        "setp.eq.b32 ph, ck, %3;\n\t"              // the label's slot: hit
-        "setp.eq.b32 pc, ck, 0;\n\t"               // empty: try to claim
+        "ld.shared.v2.b32 {ck, cv}, [%2];\n\t"
+        "setp.eq.and.b32 ph, ck, %3, pn;\n\t"      // the label's slot: hit
+        "setp.lt.and.u32 pc, ck, %5, pn;\n\t"      // empty (zeroed or an earlier vertex's): try to claim
         "@pc st.shared.b32 [%2], %3;\n\t"
-        "bar.warp.sync 0xFFFFFFFF;\n\t"
-        "mov.b32 now, 0;\n\t"
+        KV_WSYNC
         "@pc ld.shared.b32 now, [%2];\n\t"
         "setp.eq.and.b32 pd, now, %3, pc;\n\t"     // this lane's store survived: claimed
+        "@!ph mov.f32 cv, 0f00000000;\n\t"         // a claimed slot starts at 0
         "or.pred pd, pd, ph;\n\t"
         "add.rn.f32 nv, cv, %4;\n\t"
         "@pd st.shared.f32 [%2+4], nv;\n\t"
@@ -470,7 +530,7 @@ __device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, float x, bo
         "@pd mov.b32 %0, 0;\n\t"
         "}"
         : "+r"(n), "+r"(vb)
-        : "r"(addr), "r"(tg), "f"(x)
+        : "r"(addr), "r"(tg), "f"(x), "r"(epb)
         : "memory");
     need = n != 0;
     V = __uint_as_float(vb);
@@ -481,12 +541,12 @@ __device__ __forceinline__ void kv_round(uint32_t addr, uint32_t tg, float x, bo
 // probing, R5 linear continuation after kMaxRetries probes.  Called by the
 // whole warp (rounds are warp-synchronous); lanes without `need` idle.
 template <uint32_t P>
-__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint32_t i, bool need, float V) {
+__device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, uint32_t epb, float x, uint32_t i, bool need, float V) {
     constexpr uint32_t p2 = 2 * P + 1;                    // R3
     const uint32_t km = ((uint32_t)k % p2) % P;
     uint32_t di = 2 + km;
     if (di >= P) di -= P;
-    const uint32_t tg = kv_tag(k);
+    const uint32_t tg = kv_tag(k, epb);
     for (int t = 2; __any_sync(0xFFFFFFFFu, need); ++t) {
         if (t <= kMaxRetries) {
             i += di;
@@ -497,7 +557,7 @@ __device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint
         } else {
             i = i + 1 == P ? 0 : i + 1;                    // R5
         }
-        kv_round(tab + 8 * i, tg, x, need, V);
+        kv_round(tab + 8 * i, tg, epb, x, need, V);
     }
     return V;
 }
@@ -507,16 +567,16 @@ __device__ __noinline__ float kv_add_slow(uint32_t tab, int32_t k, float x, uint
 // (home + 1) inline, later probes out of line.  Returns the label's new
 // total (leaders only).  Warp-synchronous: called by all 32 lanes.
 template <uint32_t P>
-__device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, float x, bool on) {
-    const uint32_t tg = kv_tag(k);
+__device__ __forceinline__ float kv_add(uint32_t tab, int32_t k, uint32_t epb, float x, bool on) {
+    const uint32_t tg = kv_tag(k, epb);
     const uint32_t i0 = (uint32_t)k % P;
     float V = 0.0f;
     bool need = on;
-    kv_round(tab + 8 * i0, tg, x, need, V);
+    kv_round(tab + 8 * i0, tg, epb, x, need, V);
     if (__any_sync(0xFFFFFFFFu, need)) {
         const uint32_t i1 = i0 + 1 == P ? 0u : i0 + 1;
-        kv_round(tab + 8 * i1, tg, x, need, V);
-        if (__any_sync(0xFFFFFFFFu, need)) V = kv_add_slow<P>(tab, k, x, i1, need, V);
+        kv_round(tab + 8 * i1, tg, epb, x, need, V);
+        if (__any_sync(0xFFFFFFFFu, need)) V = kv_add_slow<P>(tab, k, epb, x, i1, need, V);
     }
     return V;
 }
@@ -791,7 +851,7 @@ struct GroupFetcher {
 template <bool W, int SLOTS, bool O32>
 __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, int lane, unsigned lanes_below,
                                              uint64_t row_o, uint32_t dk, int32_t vk, int32_t k0a, int32_t k0b,
-                                             float w0a, float w0b) {
+                                             float w0a, float w0b, uint32_t &ep) {
     constexpr int U = WarpCfg<SLOTS>::unroll;
     (void)U;
     const int32_t *__restrict__ lab_in = a.lab_in;
@@ -817,14 +877,20 @@ __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, i
     } else {
         auto table_row = [&](auto cap) {
             constexpr uint32_t P = decltype(cap)::value;
+            // hashtableClear: next epoch; zero the whole table when the epoch wraps
+            const uint32_t emax = NULPA_EPOCH ? (1u << (32 - a.kbits)) - 1u : 1u;
+            if (++ep > emax) {
 #pragma unroll
-            for (uint32_t q = 0; q < (P + 1) / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));   // hashtableClear
-            __syncwarp();
+                for (uint32_t q = 0; q < SLOTS / 64; ++q) sts_v4_empty(tab + 16 * (q * 32 + lane));
+                wsync();
+                ep = 1;
+            }
+            const uint32_t epb = ep << a.kbits;
             auto batch = [&](int32_t key, float w, bool eq) {
                 const unsigned grp = __match_any_sync(0xFFFFFFFFu, key);
                 const bool leader = key != kEmpty && (grp & lanes_below) == 0;
                 const float x = group_total(grp, key, w, eq);
-                const float V = kv_add<P>(tab, key, x, leader);
+                const float V = kv_add<P>(tab, key, epb, x, leader);
                 // running best (total, smallest label) as one 64-bit max
                 const uint64_t c = ((uint64_t)(__float_as_uint(V) + 1) << 32) | (uint32_t)~key;
                 const uint64_t b = ((uint64_t)bw << 32) | (uint32_t)~bk;
@@ -832,7 +898,7 @@ __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, i
                     bw = (uint32_t)(c >> 32);
                     bk = key;
                 }
-                __syncwarp();
+                wsync();
             };
             batch(k0a, w0a, eqw);
             batch(k0b, w0b, eqw);
@@ -851,7 +917,7 @@ __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, i
                     if (W && ok) xu[u] = ld_stream(pw + b + 32 * u);
                 }
 #pragma unroll
-                for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != vk) ? lab_in[iu[u]] : kEmpty;
+                for (int u = 0; u < U; ++u) qu[u] = (iu[u] >= 0 && iu[u] != vk) ? ld_label(lab_in + iu[u]) : kEmpty;
                 bool eq = true;
                 if (W) {
                     bool e = true;
@@ -949,45 +1015,50 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         ring_put(G, r1);
     }
     VRec pend = grec(F.next(ws, lane));
-    __syncwarp();
+    wsync();
     const int32_t *__restrict__ lab_in = a.lab_in;
     // row loads: entries lane and lane+32 of the row of record m
     // entry e of the CSR arrays (e = row offset + position)
     auto at = [&](uint64_t o, uint32_t k) -> uint64_t { return O32 ? (uint64_t)((uint32_t)o + k) : o + k; };
-    auto load_row = [&](const VRec &r, int32_t &ja, int32_t &jb, float &wa, float &wb) {
+    auto load_idx = [&](const VRec &r, int32_t &ja, int32_t &jb) {
         const uint32_t d = r_d(r);
-        const uint64_t e = at(r_o(r), (uint32_t)lane);
-        const int32_t *pi = a.indices + e;
+        const int32_t *pi = a.indices + at(r_o(r), (uint32_t)lane);
         ja = (uint32_t)lane < d ? ld_stream(pi) : -1;
         jb = (uint32_t)lane + 32 < d ? ld_stream(pi + 32) : -1;
+    };
+    auto load_w = [&](const VRec &r, float &wa, float &wb) {
         wa = wb = 1.0f;
         if (W) {
-            const float *pw = a.weights + e;
+            const uint32_t d = r_d(r);
+            const float *pw = a.weights + at(r_o(r), (uint32_t)lane);
             if ((uint32_t)lane < d) wa = ld_stream(pw);
             if ((uint32_t)lane + 32 < d) wb = ld_stream(pw + 32);
         }
     };
     // label gathers ("if j = i continue": the vertex's own entries are skipped)
     auto gather = [&](int32_t vk, int32_t ja, int32_t jb, int32_t &ka, int32_t &kb) {
-        ka = (ja >= 0 && ja != vk) ? lab_in[ja] : kEmpty;
-        kb = (jb >= 0 && jb != vk) ? lab_in[jb] : kEmpty;
+        ka = (ja >= 0 && ja != vk) ? ld_label(lab_in + ja) : kEmpty;
+        kb = (jb >= 0 && jb != vk) ? ld_label(lab_in + jb) : kEmpty;
     };
-    // pipeline registers: vertex n (fold) / n+1 (gathers in flight) / n+2 (row loads in flight)
+    // pipeline registers: vertex n (fold) / n+1 (gathers and weight loads in
+    // flight) / n+2 (index loads in flight)
     int32_t j0a, j0b, k0a, k0b, j1a, j1b, k1a, k1b, j2a, j2b;
-    float w0a, w0b, w1a, w1b, w2a, w2b;
+    float w0a, w0b, w1a, w1b;
     {
-        load_row(rrec_at(ring), j0a, j0b, w0a, w0b);
-        load_row(rrec_at(ring + 16), j1a, j1b, w1a, w1b);
+        load_idx(rrec_at(ring), j0a, j0b);
+        load_idx(rrec_at(ring + 16), j1a, j1b);
+        load_w(rrec_at(ring), w0a, w0b);
         gather(rrec_at(ring).r + (int32_t)a.row_begin, j0a, j0b, k0a, k0b);
     }
     uint32_t c_ch = 0, c_che = 0;
+    uint32_t ep = 0xFFFFFFFEu;                             // table epoch: the first table vertex zeroes the table
     for (uint32_t q = 0;; ++q) {                           // record groups
       if (q > 0) {
           // entering group q (groups q-1, q in the ring): group q+1 (pend)
           // goes where group q-1 was, group q+2 is requested
           ring_put(((q + 1) & 1) * G, pend);
           pend = grec(F.next(ws, lane));
-          __syncwarp();
+          wsync();
       }
       const uint32_t ring_q = ring + 16u * ((q & 1) * G);
       for (uint32_t p = 0; p < (uint32_t)G; ++p) {          // vertex n = q*G + p
@@ -995,11 +1066,15 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         const VRec rc = rrec_at(rn);
         if (rc.r < 0) goto done;                           // end record
         const uint32_t dk = r_d(rc);
-        load_row(rrec_at(rn + 32), j2a, j2b, w2a, w2b);
-        gather(rrec_at(rn + 16).r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
+        load_idx(rrec_at(rn + 32), j2a, j2b);
+        {
+            const VRec r1 = rrec_at(rn + 16);
+            gather(r1.r + (int32_t)a.row_begin, j1a, j1b, k1a, k1b);
+            load_w(r1, w1a, w1b);
+        }
         // ---- fold vertex n ----
         const int32_t vk = rc.r + (int32_t)a.row_begin;
-        const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, k0a, k0b, w0a, w0b);
+        const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, k0a, k0b, w0a, w0b, ep);
         if (accept_move(cs, rc.ci, pl)) {
             c_ch += 1;
             c_che += dk;
@@ -1015,7 +1090,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         }
         // rotate the pipeline
         j0a = j1a; j0b = j1b; k0a = k1a; k0b = k1b; w0a = w1a; w0b = w1b;
-        j1a = j2a; j1b = j2b; w1a = w2a; w1b = w2b;
+        j1a = j2a; j1b = j2b;
       }
     }
 done:
@@ -2153,6 +2228,8 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
     SweepArgs a;
     a.pl_dev = pl_dev;
     a.first = g->sweeps_since_reset == 0;
+    a.kbits = 1;
+    while (a.kbits < 31 && (INT64_C(1) << a.kbits) <= g->n_global) ++a.kbits;   // key + 1 <= n_global < 2^kbits
     a.offsets = g->offsets;
     a.indices = g->indices;
     a.weights = g->weights;

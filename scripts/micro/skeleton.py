@@ -10,16 +10,51 @@ src = r"""
 #include <torch/extension.h>
 #include <cuda_runtime.h>
 template <int MODE>
-__global__ void __launch_bounds__(256, 6) skel(const long* __restrict__ off, const int* __restrict__ idx, const float* __restrict__ wt,
-    const int* __restrict__ lab, const int* __restrict__ list, long n, int* out) {
+__global__ void __launch_bounds__(256, 8) skel(const long* __restrict__ off, const int* __restrict__ idx, const float* __restrict__ wt,
+    const int* __restrict__ lab, const int* __restrict__ list, long n, int* out, int contig) {
   const int lane = threadIdx.x & 31;
   long nw = (long)gridDim.x * 8;
   int acc = 0;
-  for (long c = (long)blockIdx.x * 8 + (threadIdx.x >> 5); c < (n + 31) / 32; c += nw) {
+  const long nc = (n + 31) / 32, gw = (long)blockIdx.x * 8 + (threadIdx.x >> 5);
+  const long c0 = contig ? gw * nc / nw : gw, c1 = contig ? (gw + 1) * nc / nw : nc, cs = contig ? 1 : nw;
+  for (long c = c0; c < c1; c += cs) {
     long t = c * 32 + lane;
     long o = 0; unsigned d = 0;
     if (t < n) { int r = list[t]; o = off[r]; d = (unsigned)(off[r + 1] - o); }
     unsigned act = __ballot_sync(~0u, d > 0);
+    if (MODE >= 3) {
+      // software-pipelined: at vertex k, index loads of k+D+1, gathers of k+D, consume k
+      constexpr int D = MODE - 2;
+      int J[D + 2][2]; int K[D + 1][2];
+      auto ldidx = [&](int k, int* jj) {
+        long ok = __shfl_sync(~0u, o, k & 31); unsigned dk = __shfl_sync(~0u, d, k & 31);
+        if (k >= 32) dk = 0;
+        jj[0] = lane < dk ? __ldcs(idx + ok + lane) : -1;
+        jj[1] = lane + 32 < dk ? __ldcs(idx + ok + 32 + lane) : -1;
+      };
+      auto gat = [&](const int* jj, int* kk) { kk[0] = jj[0] >= 0 ? lab[jj[0]] : 0; kk[1] = jj[1] >= 0 ? lab[jj[1]] : 0; };
+#pragma unroll
+      for (int s = 0; s <= D; ++s) ldidx(s, J[s]);
+#pragma unroll
+      for (int s = 0; s < D; ++s) gat(J[s], K[s]);
+      for (int k = 0; k < 32; ++k) {
+        ldidx(k + D + 1, J[D + 1]);
+        gat(J[D], K[D]);
+        acc ^= K[0][0] ^ K[0][1];
+        // rest of row k (entries 64..), unpipelined
+        long ok = __shfl_sync(~0u, o, k); unsigned dk = __shfl_sync(~0u, d, k);
+        for (unsigned b = 64; b < dk; b += 64) {
+          int j0 = b + lane < dk ? __ldcs(idx + ok + b + lane) : -1;
+          int j1 = b + 32 + lane < dk ? __ldcs(idx + ok + b + 32 + lane) : -1;
+          acc ^= (j0 >= 0 ? lab[j0] : 0) ^ (j1 >= 0 ? lab[j1] : 0);
+        }
+#pragma unroll
+        for (int s = 0; s < D; ++s) { K[s][0] = K[s + 1][0]; K[s][1] = K[s + 1][1]; }
+#pragma unroll
+        for (int s = 0; s <= D; ++s) { J[s][0] = J[s + 1][0]; J[s][1] = J[s + 1][1]; }
+      }
+      continue;
+    }
     while (act) {
       int k = __ffs(act) - 1; act &= act - 1;
       long ok = __shfl_sync(~0u, o, k); unsigned dk = __shfl_sync(~0u, d, k);
@@ -39,15 +74,18 @@ __global__ void __launch_bounds__(256, 6) skel(const long* __restrict__ off, con
   }
   if (acc == 0x12345) out[0] = acc;
 }
-void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor lab, torch::Tensor list, torch::Tensor out, int mode, int grid) {
+void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor lab, torch::Tensor list, torch::Tensor out, int mode, int grid, int contig) {
   long n = list.numel();
   auto s = at::cuda::getCurrentCUDAStream();
-  if (mode == 0) skel<0><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>());
-  else if (mode == 1) skel<1><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>());
-  else skel<2><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>());
+  if (mode == 0) skel<0><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 1) skel<1><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 2) skel<2><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 3) skel<3><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 4) skel<4><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else skel<6><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
 }
 """
-m = load_inline("skel", cpp_sources="void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor lab, torch::Tensor list, torch::Tensor out, int mode, int grid);",
+m = load_inline("skel", cpp_sources="void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor lab, torch::Tensor list, torch::Tensor out, int mode, int grid, int contig);",
                 cuda_sources="#include <ATen/cuda/CUDAContext.h>\n" + src, functions=["run"],
                 extra_cuda_cflags=["-gencode", "arch=compute_100a,code=sm_100a", "-O3"], verbose=False)
 g = synth.make("web_40m_2200m", device="cuda")
@@ -60,11 +98,13 @@ gg.run()
 labels = gg.labels().clone()
 out = torch.zeros(1, dtype=torch.int32, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-for mode, name in ((0, "stream idx+w"), (1, "+ label gather"), (2, "+ gather + 2 match_any")):
-    for grid in (148 * 6,):
+MODES = [int(x) for x in os.environ.get("SKEL_MODES", "0,1,2").split(",")]
+NAMES = {0: "stream idx+w", 1: "+ label gather", 2: "+ gather + 2 match_any", 3: "pipelined idx, gather lead 1", 4: "pipelined, gather lead 2", 6: "pipelined, gather lead 4"}
+for mode, name in [(m, NAMES[m]) for m in MODES]:
+    for grid, contig in ((148 * 4, 0), (148 * 6, 0), (148 * 8, 0), (148 * 4, 1), (148 * 8, 1)):
         ts = []
         for r in range(4):
             torch.cuda.synchronize(); e0.record()
-            m.run(g.offsets, g.indices, w, labels, rows, out, mode, grid)
+            m.run(g.offsets, g.indices, w, labels, rows, out, mode, grid, contig)
             e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
-        print(f"{name:28s} grid {grid}: {min(ts):.3f} ms", flush=True)
+        print(f"{name:28s} grid {grid} contig {contig}: {min(ts):.3f} ms", flush=True)
