@@ -41,7 +41,8 @@ namespace {
 constexpr int32_t kEmpty = -1;           // phi
 constexpr int kMaxRetries = 16;          // R5
 constexpr int kMaxIter = 64;             // counters kept per iteration
-constexpr int kCtr = 24;                 // counters per iteration
+constexpr int kCtr = 32;                 // counters per iteration
+constexpr int kCtrTScan = 24;            // counter slots 24..31: thread-bin compaction, one per wave
 constexpr int kCtrRecs = 20;             // counter slot: warp-bin frontier size
 constexpr int kCtrRecsW = 21;            // counter slot: block-bin frontier, warp-per-vertex part
 constexpr int kCtrRecsB = 22;            // counter slot: block-bin frontier, CTA-per-vertex part
@@ -435,6 +436,195 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
         }
     }
     // counters: warp sums, then one set of global atomics per CTA
+    n_act = __reduce_add_sync(0xFFFFFFFFu, n_act);
+    n_ch = __reduce_add_sync(0xFFFFFFFFu, n_ch);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        e_act += __shfl_xor_sync(0xFFFFFFFFu, e_act, o);
+        e_ch += __shfl_xor_sync(0xFFFFFFFFu, e_ch, o);
+    }
+    if ((threadIdx.x & 31) == 0 && n_act) {
+        atomicAdd(&bctr[0], (unsigned long long)n_act);
+        atomicAdd(&bctr[1], e_act);
+        atomicAdd(&bctr[2], (unsigned long long)n_ch);
+        atomicAdd(&bctr[3], e_ch);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && bctr[0]) {
+        atomicAdd(&a.ctr[1], bctr[0]);
+        atomicAdd(&a.ctr[5], bctr[1]);
+        if (bctr[2]) {
+            atomicAdd(&a.ctr[0], bctr[2]);
+            atomicAdd(&a.ctr[9], bctr[2]);
+            atomicAdd(&a.ctr[13], bctr[3]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Thread bin over a compacted frontier (asynchronous mode, bulk thread bins:
+// road / k-mer graphs, where the thread bin is the whole sweep).  k_tscan is
+// the vertex-pruning test of Algorithm 1 as a streaming
+// pass over a slice of the bin list: the unprocessed rows, in list order
+// within each CTA tile, are appended to `out` and their flags cleared ("mark
+// i as processed"); one global atomic per tile.  k_tact then gives every
+// thread 4 consecutive compacted rows (the ID-order propagation of the
+// grid-stride k_thread: vertex u sees the labels rows u-1.. of its quad
+// wrote) and issues the loads of V of them at once -- offsets, indices,
+// weights, neighbour labels -- before deciding them in order; a label
+// gathered before an earlier row of the quad moved is patched to the new
+// label (as k_warp does for its pipelined vertex).  Late sweeps of a road
+// network process a few percent of the bin: the plain grid-stride kernel
+// pays its dependent list -> flag -> offsets -> indices -> labels round
+// trips on every step of every warp; here only the active rows are visited,
+// with all their loads in flight.
+// ---------------------------------------------------------------------------
+constexpr int kTScanThreads = 256;
+__global__ void __launch_bounds__(kTScanThreads) k_tscan(SweepArgs a, const int32_t *__restrict__ list, int64_t n,
+                                                         int32_t *__restrict__ out, unsigned long long *count) {
+    constexpr int NW = kTScanThreads / 32;
+    __shared__ uint32_t s_w[NW];
+    __shared__ unsigned long long s_base;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int64_t tile = (int64_t)blockIdx.x * kTScanThreads * 4; tile < n; tile += (int64_t)gridDim.x * kTScanThreads * 4) {
+        const int64_t q = tile + 4 * (int64_t)threadIdx.x;
+        int32_t r[4] = {-1, -1, -1, -1};
+        if (q + 3 < n) {
+            const int4 v4 = *reinterpret_cast<const int4 *>(list + q);     // slices start on 16-byte boundaries
+            r[0] = v4.x; r[1] = v4.y; r[2] = v4.z; r[3] = v4.w;
+        } else {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) r[u] = q + u < n ? list[q + u] : -1;
+        }
+        bool act[4];
+        uint32_t c = 0;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            act[u] = r[u] >= 0 && a.flag_in[r[u] + a.row_begin] != 0;
+            c += act[u];
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (act[u]) a.flag_in[r[u] + a.row_begin] = 0;          // mark i as processed
+        uint32_t incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+            if (lane >= o) incl += t;
+        }
+        if (lane == 31) s_w[wid] = incl;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t tot = 0;
+#pragma unroll
+            for (int w = 0; w < NW; ++w) tot += s_w[w];
+            s_base = tot ? atomicAdd(count, (unsigned long long)tot) : 0;
+        }
+        __syncthreads();
+        unsigned long long pos = s_base + incl - c;
+        for (int w = 0; w < wid; ++w) pos += s_w[w];
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (act[u]) out[pos++] = r[u];
+        __syncthreads();                                          // s_w / s_base reused by the next tile
+    }
+}
+
+// V rows of a quad have their loads in flight together (V = 4 for degrees
+// <= 4: road; 2 above)
+template <bool W, int MAXD, int V>
+__global__ void __launch_bounds__(kThreadThreads) k_tact(SweepArgs a, const int32_t *__restrict__ rows,
+                                                         const unsigned long long *__restrict__ count) {
+    __shared__ unsigned long long bctr[4];
+    if (threadIdx.x < 4) bctr[threadIdx.x] = 0;
+    __syncthreads();
+    const int64_t n = (int64_t)*count;
+    uint32_t n_act = 0, n_ch = 0;
+    unsigned long long e_act = 0, e_ch = 0;
+    const int pl = sweep_pl(a);
+    for (int64_t q = (int64_t)blockIdx.x * kThreadThreads + threadIdx.x; 4 * q < n; q += (int64_t)gridDim.x * kThreadThreads) {
+#pragma unroll
+        for (int h = 0; h < 4; h += V) {
+            // rows of this group that moved (-2: did not) and their new labels;
+            // earlier groups wrote their labels before this group's loads
+            int32_t vmov[V], cmov[V];
+            int32_t v[V], ci[V], lab[V][MAXD], jj[V][MAXD];
+            float w[V][MAXD];
+            int64_t o[V];
+            uint32_t deg[V];
+#pragma unroll
+            for (int u = 0; u < V; ++u) {
+                const int64_t e = 4 * q + h + u;
+                v[u] = -1;
+                deg[u] = 0;
+                o[u] = 0;
+                ci[u] = 0;
+                vmov[u] = -2;
+                cmov[u] = 0;
+                if (e < n) {
+                    const int32_t r = rows[e];
+                    v[u] = (int32_t)(r + a.row_begin);
+                    o[u] = a.offsets[r];
+                    deg[u] = (uint32_t)(a.offsets[r + 1] - o[u]);
+                    ci[u] = a.lab_in[v[u]];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < V; ++u)
+#pragma unroll
+                for (int k = 0; k < MAXD; ++k) {
+                    jj[u][k] = -1;
+                    lab[u][k] = kEmpty;
+                    w[u][k] = 0.0f;
+                    if (k < (int)deg[u]) {
+                        jj[u][k] = a.indices[o[u] + k];
+                        if (W) w[u][k] = a.weights[o[u] + k];
+                    }
+                }
+#pragma unroll
+            for (int u = 0; u < V; ++u)
+#pragma unroll
+                for (int k = 0; k < MAXD; ++k)
+                    if (jj[u][k] >= 0 && jj[u][k] != v[u]) {        // "if j = i continue"
+                        lab[u][k] = a.lab_in[jj[u][k]];
+                        if (!W) w[u][k] = 1.0f;
+                    }
+#pragma unroll
+            for (int u = 0; u < V; ++u) {
+                if (v[u] < 0) continue;
+                // labels gathered before an earlier row of the group moved
+#pragma unroll
+                for (int p = 0; p < u; ++p)
+#pragma unroll
+                    for (int k = 0; k < MAXD; ++k)
+                        if (jj[u][k] == vmov[p]) lab[u][k] = cmov[p];
+                TieOrder to;
+                uint64_t best = 0;
+#pragma unroll
+                for (int k = 0; k < MAXD; ++k) {
+                    if (lab[u][k] == kEmpty) continue;
+                    float s = 0.0f;
+#pragma unroll
+                    for (int m = 0; m < MAXD; ++m) s = __fadd_rn(s, lab[u][m] == lab[u][k] ? w[u][m] : 0.0f);
+                    const uint64_t c = pack_cand(s, lab[u][k], to);
+                    best = c > best ? c : best;
+                }
+                const int32_t cs = best ? cand_label(best, to) : kEmpty;
+                n_act += 1;
+                e_act += deg[u];
+                if (accept_move(cs, ci[u], pl)) {
+                    a.lab_out[v[u]] = cs;
+                    n_ch += 1;
+                    e_ch += deg[u];
+#pragma unroll
+                    for (int k = 0; k < MAXD; ++k)
+                        if (jj[u][k] >= 0) a.flag_out[jj[u][k]] = 1;
+                    vmov[u] = v[u];
+                    cmov[u] = cs;
+                }
+            }
+        }
+    }
     n_act = __reduce_add_sync(0xFFFFFFFFu, n_act);
     n_ch = __reduce_add_sync(0xFFFFFFFFu, n_ch);
 #pragma unroll
@@ -1802,6 +1992,7 @@ struct nulpa_graph {
     bool bins_built = false;
     int32_t *bin_list[4] = {nullptr, nullptr, nullptr, nullptr};
     void *wrecs = nullptr;          // warp-bin frontier records (VRec [bin_n[1]])
+    int32_t *trows = nullptr;       // thread-bin compacted frontier (rows [bin_n[0]]), k_tscan / k_tact
     unsigned long long *wranges = nullptr;   // SCHED_STEAL: one {next, end} group range per k_warp warp
     double locality = 0.0;          // share of sampled CSR entries j with |j - i| <= kNear (k_locality)
     void *brecs = nullptr;          // block-bin frontier records (VRec [2 * bin_n[2]]: warp part | CTA part)
@@ -1906,6 +2097,8 @@ void free_bins(nulpa_graph *g) {
     free_loop(g);
     dfree(g->wrecs);
     g->wrecs = nullptr;
+    dfree(g->trows);
+    g->trows = nullptr;
     dfree(g->wranges);
     g->wranges = nullptr;
     dfree(g->brecs);
@@ -2071,6 +2264,9 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CHECK(dalloc(&g->bin_list[b], (size_t)ht[b]));
         L.l[b] = g->bin_list[b];
     }
+    // thread-bin compacted frontier (bulk bins of low degree; allocated here,
+    // not in the sweep, which the device loop captures into a CUDA graph)
+    if (2 * g->bin_e[0] >= g->M && g->bin_maxdeg[0] <= 8) CHECK(dalloc(&g->trows, (size_t)g->bin_n[0]));
     if (nb > 0) {
         k_bin_scatter<<<(unsigned)nb, kBinTile, 0, g->stream>>>(g->offsets, n, t1, t2, t3, counts, L);
         CU(cudaGetLastError());
@@ -2188,6 +2384,10 @@ int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
 #define NULPA_THREAD_WAVES 8
 #endif
 constexpr int kThreadWaves = NULPA_THREAD_WAVES;
+static_assert(kThreadWaves <= kCtr - kCtrTScan, "one compaction counter per wave");
+#ifndef NULPA_TCOMPACT
+#define NULPA_TCOMPACT 1                 // asynchronous bulk thread bins: compacted frontier
+#endif
 template <bool SYNC, bool W>
 int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const int64_t n = g->bin_n[0];
@@ -2201,6 +2401,9 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
     const bool bulk = 2 * g->bin_e[0] >= g->M;
     int64_t waves = SYNC || !bulk ? 1 : (kThreadWaves * per_step + n - 1) / std::max<int64_t>(n, 1);
     waves = std::max<int64_t>(1, std::min<int64_t>({waves, (int64_t)kThreadWaves, n / 1024}));
+    // asynchronous bulk bins of low degree: compacted frontier (k_tscan + k_tact)
+    const bool compact = NULPA_TCOMPACT && !SYNC && bulk && md <= 8;
+    if (compact && !g->trows) return fail(NULPA_ESTATE, "thread-bin frontier not allocated");
     for (int64_t w = 0; w < waves; ++w) {
         // slice bounds on multiples of 4 entries (k_thread reads the list 16 bytes at a time)
         const int64_t b0 = (n * w / waves) & ~INT64_C(3), b1 = w + 1 == waves ? n : (n * (w + 1) / waves) & ~INT64_C(3);
@@ -2208,6 +2411,16 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
         const int32_t *list = g->bin_list[0] + b0;
         const int grid = bulk ? grid_for((m + 3) / 4, kThreadThreads, num_sms() * 8)   // 4 entries per thread and step
                               : grid_for(m, kThreadThreads, num_sms() * 32);
+        if (compact) {
+            unsigned long long *cnt = a.ctr + kCtrTScan + w;
+            k_tscan<<<grid_for(m, 4 * kTScanThreads, num_sms() * 8), kTScanThreads, 0, g->stream>>>(a, list, m, g->trows, cnt);
+            if (md <= 4)
+                k_tact<W, 4, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->trows, cnt);
+            else
+                k_tact<W, 8, 2><<<grid, kThreadThreads, 0, g->stream>>>(a, g->trows, cnt);
+            CU(cudaGetLastError());
+            continue;
+        }
         if (md <= 4)
             k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
         else if (md <= 8)
@@ -2218,7 +2431,7 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
             k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
         CU(cudaGetLastError());
     }
-    g->stats.launches[0] += (int)waves - 1;
+    g->stats.launches[0] += (int)waves * (compact ? 2 : 1) - 1;
     return NULPA_OK;
 }
 
