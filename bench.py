@@ -318,7 +318,11 @@ def run_ours(args):
     # region when its events there are its own (thread, warp bins), else
     # from the serial runs.
     eff = effective_params(params)
-    overlapped = (2, 3) if eff["bin_order"] == 3 else ()
+    order = eff["bin_order"]
+    if order == 4:      # auto (nulpa.h): 3 when the warp bin holds >= 2/3 of the CSR entries, else 1
+        order = 3 if 3 * stats[-1]["bin_edges"][1] >= 2 * M else 1
+    eff["bin_order_resolved"] = order
+    overlapped = (2, 3) if order == 3 else ()
     tot_ms = [sum(s["kernel_ms"][b] for s in stats) for b in range(4)]
     ser = [gg.run(**{**params, "bin_order": 1}) for _ in range(3)]
     bins_serial = [round(sum(s["kernel_ms"][b] for s in ser) / len(ser), 3) for b in range(4)]

@@ -68,13 +68,14 @@ typedef struct nulpa_params {
                                     star "ties broken by smallest label"; "the
                                     first label with the highest associated weight").  Any other
                                     value is rejected with NULPA_EINVAL                          */
-    int32_t bin_order;           /* 3 (default): thread bin, then the warp bin on a
+    int32_t bin_order;           /* 4 (default, auto): 3 if the warp bin holds >= 2/3 of the
+                                    CSR entries, else 1.  3: thread bin, then the warp bin on a
                                     high-priority stream and block + giant on a low-priority
                                     stream released after the warp-bin frontier (they fill the
-                                    warp bin's tail: +5% at first_sweep_block 192); 1: thread,
-                                    warp, block, giant bins in that order within a sweep (hubs
-                                    last); 0: giant, block, warp, thread; 2: block + giant on a
-                                    second stream, concurrent with thread + warp              */
+                                    warp bin's tail); 1: thread, warp, block, giant bins in
+                                    that order within a sweep (hubs last); 0: giant, block,
+                                    warp, thread; 2: block + giant on a second stream,
+                                    concurrent with thread + warp                             */
     int32_t wide_degree;         /* within the block bin: degree < this -> one warp per vertex
                                     with a warp-private 1023-slot shared-memory table (load
                                     <= 1/2 at 512); degree >= this -> one CTA per vertex.

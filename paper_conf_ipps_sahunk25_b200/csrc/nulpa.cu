@@ -915,7 +915,10 @@ __global__ void __launch_bounds__(kFrontThreads) k_frontier(SweepArgs a, const i
 //    consecutive groups from a global counter.
 //  * SCHED_STRIDED (K = 1): groups w, w + nw, ...
 // ---------------------------------------------------------------------------
-constexpr int kWarpWarps = 8;            // warps per CTA
+#ifndef NULPA_WARP_WARPS
+#define NULPA_WARP_WARPS 8
+#endif
+constexpr int kWarpWarps = NULPA_WARP_WARPS;   // warps per CTA
 #ifndef NULPA_WARP_CTAS
 #define NULPA_WARP_CTAS 4
 #endif
@@ -2356,7 +2359,7 @@ int validate_params(const nulpa_params &p) {
     if (p.block_degree < p.switch_degree || p.block_degree > 256)
         return fail(NULPA_EINVAL, "block_degree must be in [switch_degree, 256] (warp tables hold 255 slots)");
     if (p.tie_rule != NULPA_TIE_SMALLEST) return fail(NULPA_EINVAL, "tie_rule must be NULPA_TIE_SMALLEST (0): ties go to the smallest label (R6)");
-    if (p.bin_order < 0 || p.bin_order > 3) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2 or 3");
+    if (p.bin_order < 0 || p.bin_order > 4) return fail(NULPA_EINVAL, "bin_order must be 0, 1, 2, 3 or 4");
     if (p.first_sweep_block < 0 || p.first_sweep_block > 1024 || p.sweep_block < 0 || p.sweep_block > 1024)
         return fail(NULPA_EINVAL, "first_sweep_block and sweep_block must be in [0, 1024]");
     if (p.wide_degree < 1 || p.wide_degree > 1024)   // distinct labels <= D <= 1023 = p1 (R5 always finds a slot)
@@ -2547,6 +2550,12 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(2, 1));
         return NULPA_OK;
     };
+    // bin_order 4 (auto): 3 when the warp bin holds >= 2/3 of the CSR entries
+    // (web, SBM: the block + giant bins fill its tail), else 1 (social graphs:
+    // block + giant bins are ~half the entries and would wait for the warp
+    // bin's CTAs on the low-priority stream; measured R-MAT 4M/70M 17.0 ->
+    // 19.8e9 edges/s with 1)
+    const int order = p.bin_order == 4 ? (3 * g->bin_e[1] >= 2 * g->M ? 3 : 1) : p.bin_order;
     bool mid_fork = false;                        // bin_order 3: record ev_mid after the warp-bin frontier
     auto run_warp = [&]() -> int {
         const int64_t n = g->bin_n[1];
@@ -2592,12 +2601,12 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         CHECK(rec(0, 1));
         return NULPA_OK;
     };
-    if (p.bin_order == 0) {
+    if (order == 0) {
         CHECK(run_giant());
         CHECK(run_block());
         CHECK(run_warp());
         CHECK(run_thread());
-    } else if (p.bin_order == 3) {
+    } else if (order == 3) {
         // thread bin on the caller's stream; warp bin on a high-priority
         // stream; block + giant bins on a low-priority side stream released
         // after the warp-bin frontier: k_warp's CTAs take every SM's register
@@ -2630,7 +2639,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         cs = g->stream;
         CU(cudaStreamWaitEvent(g->stream, g->ev_join, 0));
         CU(cudaStreamWaitEvent(g->stream, g->ev_join2, 0));
-    } else if (p.bin_order == 2) {
+    } else if (order == 2) {
         // block + giant bins on a side stream, concurrent with thread + warp:
         // their latency-bound CTAs fill the SMs the warp bin leaves idle
         if (!g->side) {
@@ -2838,7 +2847,7 @@ void nulpa_default_params(nulpa_params *p) {
     p->reset = 1;
     p->timing = 0;
     p->tie_rule = NULPA_TIE_SMALLEST;
-    p->bin_order = 3;
+    p->bin_order = 4;
     p->wide_degree = 512;
     p->first_sweep_block = 0;
     p->sweep_block = 4;

@@ -22,9 +22,38 @@ __global__ void __launch_bounds__(256, MODE >= 3 ? 4 : 8) skel(const long* __res
     long o = 0; unsigned d = 0;
     if (t < n) { int r = list[t]; o = off[r]; d = (unsigned)(off[r + 1] - o); }
     unsigned act = __ballot_sync(~0u, d > 0);
+    if (MODE == 7 || MODE == 8) {
+      // chunk-pipelined: the sequence of 64-entry chunks of the 32 rows
+      // (MODE 8: entries past 64 skipped -- upper bound), loads of chunk
+      // c+2, gathers of chunk c+1, consume chunk c
+      auto nch = [&](int k) -> int { unsigned dk = __shfl_sync(~0u, d, k & 31); return k >= 32 ? 1 : (MODE == 8 ? 1 : (int)max(1u, (dk + 63) / 64)); };
+      auto ldc = [&](int k, int c, int* jj) {
+        long ok = __shfl_sync(~0u, o, k & 31); unsigned dk = __shfl_sync(~0u, d, k & 31);
+        if (k >= 32) dk = 0;
+        unsigned b = 64u * c;
+        jj[0] = b + lane < dk ? __ldcs(idx + ok + b + lane) : -1;
+        jj[1] = b + 32 + lane < dk ? __ldcs(idx + ok + b + 32 + lane) : -1;
+      };
+      auto gat = [&](const int* jj, int* kk) { kk[0] = jj[0] >= 0 ? lab[jj[0]] : 0; kk[1] = jj[1] >= 0 ? lab[jj[1]] : 0; };
+      // stage positions (row, chunk)
+      int k0 = 0, c0 = 0;
+      int k1 = k0, c1 = c0; if (++c1 >= nch(k1)) { ++k1; c1 = 0; }
+      int k2 = k1, c2 = c1; if (++c2 >= nch(k2)) { ++k2; c2 = 0; }
+      int J0[2], J1[2], J2[2], K0[2], K1[2];
+      ldc(k0, c0, J0); ldc(k1, c1, J1); gat(J0, K0);
+      while (k0 < 32) {
+        ldc(k2, c2, J2);
+        gat(J1, K1);
+        acc ^= K0[0] ^ K0[1];
+        k0 = k1; c0 = c1; k1 = k2; c1 = c2;
+        if (++c2 >= nch(k2)) { ++k2; c2 = 0; }
+        J0[0] = J1[0]; J0[1] = J1[1]; J1[0] = J2[0]; J1[1] = J2[1]; K0[0] = K1[0]; K0[1] = K1[1];
+      }
+      continue;
+    }
     if (MODE >= 3) {
       // software-pipelined: at vertex k, index loads of k+D+1, gathers of k+D, consume k
-      constexpr int D = MODE >= 3 ? MODE - 2 : 1;
+      constexpr int D = MODE >= 3 && MODE <= 6 ? MODE - 2 : 1;
       int J[D + 2][2]; int K[D + 1][2];
       auto ldidx = [&](int k, int* jj) {
         long ok = __shfl_sync(~0u, o, k & 31); unsigned dk = __shfl_sync(~0u, d, k & 31);
@@ -82,6 +111,8 @@ void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor l
   else if (mode == 2) skel<2><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else if (mode == 3) skel<3><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else if (mode == 4) skel<4><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 7) skel<7><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 8) skel<8><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else skel<6><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
 }
 """
@@ -99,7 +130,7 @@ labels = gg.labels().clone()
 out = torch.zeros(1, dtype=torch.int32, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 MODES = [int(x) for x in os.environ.get("SKEL_MODES", "0,1,2").split(",")]
-NAMES = {0: "stream idx+w", 1: "+ label gather", 2: "+ gather + 2 match_any", 3: "pipelined idx, gather lead 1", 4: "pipelined, gather lead 2", 6: "pipelined, gather lead 4"}
+NAMES = {0: "stream idx+w", 1: "+ label gather", 2: "+ gather + 2 match_any", 3: "pipelined idx, gather lead 1", 4: "pipelined, gather lead 2", 6: "pipelined, gather lead 4", 7: "chunk-pipelined lead 1", 8: "first 64 entries only (bound)"}
 for mode, name in [(m, NAMES[m]) for m in MODES]:
     for grid, contig in [(g, c) for g, c in ((148 * 4, 0), (148 * 6, 0), (148 * 8, 0), (148 * 4, 1), (148 * 8, 1)) if mode < 3 or g == 148 * 4]:
         ts = []
