@@ -44,20 +44,36 @@ if binname == "warp":
     kernels = ["k_frontier", "k_warp"]
     extra = {"k_warp_per_launch": [dram(w) for w in main], "k_frontier_per_launch": [dram(f) for f in front]}
 elif binname == "block":
-    # per sweep: the block-bin k_frontier (the one before a k_warp<..., 1024, ...>), the wide k_warp, k_block
-    wide = [k for k in ids if "k_warp" in name[k] and ", 1024" in name[k]]
-    front = [ids[ids.index(k) - 1] for k in wide]
-    blk = [next(x for x in ids[ids.index(k):] if "k_block" in name[x]) for k in wide]
-    assert all("k_frontier" in name[f] for f in front)
-    b = [dram(f) + dram(w) + dram(c) for f, w, c in zip(front, wide, blk)]
-    kernels = ["k_frontier", "k_warp<1024>", "k_block"]
-    extra = {"k_block_per_launch": [dram(c) for c in blk], "k_warp_wide_per_launch": [dram(w) for w in wide]}
+    # per sweep: the block-bin k_frontier (the one right before a k_block launch) and the k_block
+    # launches that follow it (4-warp TMA k_block below wide_degree, 8-warp above)
+    front = [k for i, k in enumerate(ids[:-1]) if "k_frontier" in name[k] and "k_block" in name[ids[i + 1]]]
+    blks = []
+    for f in front:
+        j = ids.index(f) + 1
+        bl = []
+        while j < len(ids) and "k_block" in name[ids[j]]:
+            bl.append(ids[j])
+            j += 1
+        blks.append(bl)
+    b = [dram(f) + sum(dram(c) for c in bl) for f, bl in zip(front, blks)]
+    kernels = ["k_frontier", "k_block"]
+    extra = {"k_block_per_sweep": [sum(dram(c) for c in bl) for bl in blks]}
 else:
-    # thread bin: every k_thread launch of a sweep (several waves on small bulk bins)
+    # thread bin: every k_thread launch of a sweep (synchronous mode, thin bins), or the
+    # compacted path's k_tscan + k_tact pairs (asynchronous bulk bins; one wave per sweep
+    # at full size)
     main = [k for k in ids if "k_thread" in name[k]]
-    b = [dram(k) for k in main]
-    kernels = ["k_thread"]
-    extra = {}
+    if main:
+        b = [dram(k) for k in main]
+        kernels = ["k_thread"]
+        extra = {}
+    else:
+        scan = [k for k in ids if "k_tscan" in name[k]]
+        act = [ids[ids.index(k) + 1] for k in scan]
+        assert all("k_tact" in name[k] for k in act), [name[k] for k in act]
+        b = [dram(x) + dram(y) for x, y in zip(scan, act)]
+        kernels = ["k_tscan", "k_tact"]
+        extra = {"k_tscan_per_launch": [dram(x) for x in scan], "k_tact_per_launch": [dram(y) for y in act]}
 out_path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "traffic.json")
 db = json.load(open(out_path)) if os.path.exists(out_path) else {}
 if "workload" in db:          # round-1 single-entry format
