@@ -105,7 +105,19 @@ def algorithmic_bytes(st, b, weighted, it=None):
     return v * 18 + e * (12 if weighted else 8) + c * 4 + ce * 1
 
 
-KERNELS = {0: "k_thread", 1: "k_frontier + k_warp", 2: "k_frontier + k_warp<1024> + k_block", 3: "k_giant_*"}
+KERNELS = {0: "k_thread", 1: "k_frontier + k_warp", 2: "k_frontier + k_block", 3: "k_giant_*"}
+
+
+def kernel_name(b, g, eff, M):
+    """The kernels of bin b under the effective parameters (nulpa.cu
+    launch_thread_bin: an asynchronous thread bin holding >= half of the CSR
+    entries with degrees <= 8 runs as k_tscan + k_tact)."""
+    if b == 0 and eff["mode"] == "async":
+        deg = g.offsets[1:] - g.offsets[:-1]
+        tb = deg < eff["switch_degree"]
+        if int(tb.sum()) and 2 * int(deg[tb].sum()) >= M and int(deg[tb].max()) <= 8:
+            return "k_tscan + k_tact"
+    return KERNELS[b]
 
 
 class Clocks:
@@ -353,7 +365,7 @@ def run_ours(args):
             traffic = t["dram_bytes_per_sweep"]
     sweeps = sum(s["iterations"] for s in src_runs)
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": f"{KERNELS[dom]} (bin {BINS[dom]})",
+            "frac": round(achieved / peak, 4), "traffic": traffic, "kernel": f"{kernel_name(dom, g, eff, M)} (bin {BINS[dom]})",
             "algorithmic_bytes_per_sweep": int(byts / max(1, sweeps)),
             "traffic_source": "profiles/traffic.json (ncu, per sweep of the bin's kernels)" if traffic else None,
             "peak_source": peak_src,
