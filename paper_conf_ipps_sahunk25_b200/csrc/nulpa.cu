@@ -274,53 +274,20 @@ __device__ __forceinline__ bool accept_move(int32_t cstar, int32_t ci, int pickl
 #ifndef NULPA_STREAM_LOAD
 #define NULPA_STREAM_LOAD 2              // 0: ld.global.cs (evict-first); 1: ld.global.nc; 2: plain ld.global
 #endif
-#ifndef NULPA_GATHER_POLICY
-#define NULPA_GATHER_POLICY 0            // label gathers C[j]: 0 plain; 1 L2 evict_last (fraction 1); 2 evict_last (fraction 0.5)
-#endif
-// 32-bit loads with an L2 cache-policy hint (createpolicy + ld.global.L2::cache_hint)
-__device__ __forceinline__ uint64_t l2_policy_evict_first() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ uint64_t l2_policy_evict_last(float f) {
-    uint64_t p;
-    if (f >= 1.0f) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    else asm("createpolicy.fractional.L2::evict_last.b64 %0, 0.5;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ int32_t ld_hint(const int32_t *p, uint64_t pol) {
-    int32_t v;
-    asm volatile("ld.global.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-    return v;
-}
-__device__ __forceinline__ float ld_hint(const float *p, uint64_t pol) {
-    float v;
-    asm volatile("ld.global.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
-    return v;
-}
 template <typename T>
 __device__ __forceinline__ T ld_stream(const T *p) {
 #if NULPA_STREAM_LOAD == 0
     return __ldcs(p);
 #elif NULPA_STREAM_LOAD == 1
     return __ldg(p);
-#elif NULPA_STREAM_LOAD == 3
-    return ld_hint(p, l2_policy_evict_first());
 #else
     return *p;
 #endif
 }
-// a label gather C[j]
-__device__ __forceinline__ int32_t ld_label(const int32_t *p) {
-#if NULPA_GATHER_POLICY == 1
-    return ld_hint(p, l2_policy_evict_last(1.0f));
-#elif NULPA_GATHER_POLICY == 2
-    return ld_hint(p, l2_policy_evict_last(0.5f));
-#else
-    return *p;
-#endif
-}
+// a label gather C[j] (L2 evict_last / evict_normal cache policies on the
+// gathers, and evict_first on the CSR streams, measured neutral or slower:
+// DESIGN.md experiments)
+__device__ __forceinline__ int32_t ld_label(const int32_t *p) { return *p; }
 
 // CSR indices / weights are streamed once per sweep (ld_stream).  Evict-first
 // loads (ld.global.cs), meant to keep them from pushing the gathered label
