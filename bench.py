@@ -34,6 +34,7 @@ CONTEXT = {   # the paper's A100 numbers nearest each workload (context, not tar
     "web_40m_2200m": "paper: 3.0e9 edges/s on it-2004 (2.19B edges) on one A100 (PAPER.md:501)",
     "rmat_4m_70m": "paper Table 1 social graphs (com-LiveJournal 4M / 69M, PAPER.md:456-458)",
     "road_50m_110m": "paper Table 1 road graphs (europe_osm 51M / 108M, PAPER.md:459-461)",
+    "kmer_171m_360m": "paper Table 1 protein k-mer graphs (kmer_A2a 171M / 361M, PAPER.md:462-464)",
     "sbm_1m_20m": "planted-partition SBM (north star quality config; no paper number)",
 }
 BINS = ("thread", "warp", "block", "giant")
@@ -191,8 +192,9 @@ class Clocks:
 # ---------------------------------------------------------------------------
 def oracle_sample(args):
     """A bounded sample of the workload for the oracle: a web graph of
-    --cpu-sample vertices from the same generator (the full config for the
-    smaller workloads), weights as in the timed run."""
+    --cpu-sample vertices or a 20M-vertex k-mer graph from the same
+    generator (the full config for the smaller workloads), weights as in the
+    timed run."""
     import numpy as np
     import torch
     import oracle
@@ -202,6 +204,11 @@ def oracle_sample(args):
         dev = "cuda" if torch.cuda.is_available() else "cpu"
         g = synth.web(n=n, seed=args.seed + 1, device=dev).to("cpu")
         sample = f"synth.web(n={n}) web-like graph, {g.M} CSR entries (same generator as the workload)"
+    elif args.config.startswith("kmer"):
+        nk = 20_000_000
+        dev = "cuda" if torch.cuda.is_available() else "cpu"
+        g = synth.kmer(n=nk, seed=args.seed + 1, device=dev).to("cpu")
+        sample = f"synth.kmer(n={nk}) k-mer-like graph, {g.M} CSR entries (same generator as the workload)"
     else:
         g = make_graph(args, "cpu")
         sample = f"the full {args.config} workload"

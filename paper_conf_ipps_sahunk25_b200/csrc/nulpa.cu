@@ -1110,7 +1110,6 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
     k_warp(SweepArgs a, const VRec *__restrict__ recs, const unsigned long long *__restrict__ count, int bin,
            WarpSched ws) {
     constexpr int NWARP = WarpCfg<SLOTS>::warps;
-    constexpr int U = WarpCfg<SLOTS>::unroll;
     constexpr int G = WarpCfg<SLOTS>::group;
     constexpr uint32_t RING = 2 * G;
     static_assert(G >= 1 && G <= 32 && (G & (G - 1)) == 0, "group size: power of two <= 32");

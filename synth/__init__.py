@@ -421,6 +421,8 @@ CONFIGS = {
     "rmat_4m_70m": dict(fn="rmat", kw=dict(scale=22, edge_factor=8.8)),
     "road_50m_110m": dict(fn="road", kw=dict(R=1600, mean_chain=9.5)),
     "web_40m_2200m": dict(fn="web", kw=dict(n=40_000_000)),
+    # north star "k-mer workloads": kmer_A2a-shaped (171M / 361M)
+    "kmer_171m_360m": dict(fn="kmer", kw=dict(n=171_000_000)),
 }
 
 

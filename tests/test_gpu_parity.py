@@ -206,6 +206,48 @@ def test_async_sweep_invariants(gname, bins):
         C = C2
 
 
+@pytest.mark.parametrize("gname", ["road", "kmer"])
+@pytest.mark.parametrize("weighted", [False, True])
+def test_compacted_thread_bin_sweep(gname, weighted):
+    """The asynchronous bulk thread bin of degree <= 8 (road, k-mer) runs as
+    k_tscan + k_tact over a compacted frontier (nulpa.cu).  From a random
+    mid-run state (30% of the vertices unprocessed): exactly the unprocessed
+    vertices are processed (Algorithm 1) and no other label
+    moves; every moved label is an own/neighbour label; afterwards a vertex
+    is unprocessed iff one of its neighbours moved (line 348: processed
+    vertices are cleared first, then marked); dN counts the moves."""
+    # large enough for one k_tscan/k_tact launch per sweep (bins spanning
+    # fewer than 8 grid-stride steps run in 8 ordered slices, and a later
+    # slice processes vertices an earlier one marked)
+    g = (synth.road(R=760, mean_chain=9.5, seed=5, weighted=weighted, device="cuda") if gname == "road"
+         else synth.kmer(n=10_000_000, seed=6, weighted=weighted, device="cuda")).to("cpu")
+    assert g.N > 9_800_000
+    h = host(g)
+    assert 2 * int(g.degrees()[g.degrees() < 16].sum()) >= g.M and int(g.degrees().max()) <= 8
+    gg = to_gpu(g)
+    rng = np.random.default_rng(11)
+    C0 = (np.arange(g.N) // 7 * 7).astype(np.int32)          # labels constant on blocks of 7 IDs,
+    pick = rng.random(g.N) < 0.2                               # 20% relabelled to a random block
+    C0[pick] = (rng.integers(0, g.N, int(pick.sum())) // 7 * 7).astype(np.int32)
+    U0 = (rng.random(g.N) < 0.3).astype(np.uint8)
+    gg.set_labels(torch.from_numpy(C0).cuda(), torch.from_numpy(U0).cuda())
+    before = gg.stats()["vertices_processed"][0]
+    dn = gg.sweep(False, mode=nl.ASYNC)
+    C1 = gg.labels(device=False).numpy()
+    U1 = gg.flags(device=False).numpy()
+    assert gg.stats()["vertices_processed"][0] - before == int(U0.sum())
+    moved = C1 != C0
+    assert dn == int(moved.sum())
+    assert not (moved & (U0 == 0)).any(), "a vertex that was not unprocessed moved"
+    src = np.repeat(np.arange(g.N), np.diff(h.offsets))
+    j = h.indices
+    ok = (src != j) & ((C0[j] == C1[src]) | (C1[j] == C1[src]))       # an own/neighbour label
+    assert (np.bincount(src[ok], minlength=g.N)[moved] > 0).all(), "a vertex took a label no neighbour had"
+    marked = np.zeros(g.N, dtype=bool)
+    marked[h.indices[moved[src]]] = True
+    assert np.array_equal(U1.astype(bool), marked)
+
+
 @pytest.mark.parametrize("gname", ["sbm", "web", "rmat", "road", "kmer", "hub"])
 @pytest.mark.parametrize("weighted", [False, True])
 def test_async_quality_vs_oracle(gname, weighted):
