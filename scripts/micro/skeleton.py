@@ -51,6 +51,16 @@ __global__ void __launch_bounds__(256, MODE >= 3 ? 4 : 8) skel(const long* __res
       }
       continue;
     }
+    if (MODE == 9 && c + cs < c1) {
+      // bulk L2 prefetch of the NEXT chunk's CSR index span (one instruction)
+      if (lane == 0) {
+        long tn = (c + cs) * 32;
+        int r0 = list[tn], r1 = list[min(tn + 31, n - 1)];
+        long b0 = off[r0] & ~3L, b1 = (off[r1 + 1] + 3) & ~3L;
+        unsigned bytes = (unsigned)((b1 - b0) * 4);
+        if (bytes >= 16) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(idx + b0), "r"(bytes) : "memory");
+      }
+    }
     if (MODE >= 3) {
       // software-pipelined: at vertex k, index loads of k+D+1, gathers of k+D, consume k
       constexpr int D = MODE >= 3 && MODE <= 6 ? MODE - 2 : 1;
@@ -112,6 +122,7 @@ void run(torch::Tensor off, torch::Tensor idx, torch::Tensor wt, torch::Tensor l
   else if (mode == 3) skel<3><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else if (mode == 4) skel<4><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else if (mode == 7) skel<7><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
+  else if (mode == 9) skel<9><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else if (mode == 8) skel<8><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
   else skel<6><<<grid, 256, 0, s>>>(off.data_ptr<long>(), idx.data_ptr<int>(), wt.data_ptr<float>(), lab.data_ptr<int>(), list.data_ptr<int>(), n, out.data_ptr<int>(), contig);
 }
@@ -130,7 +141,7 @@ labels = gg.labels().clone()
 out = torch.zeros(1, dtype=torch.int32, device="cuda")
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 MODES = [int(x) for x in os.environ.get("SKEL_MODES", "0,1,2").split(",")]
-NAMES = {0: "stream idx+w", 1: "+ label gather", 2: "+ gather + 2 match_any", 3: "pipelined idx, gather lead 1", 4: "pipelined, gather lead 2", 6: "pipelined, gather lead 4", 7: "chunk-pipelined lead 1", 8: "first 64 entries only (bound)"}
+NAMES = {0: "stream idx+w", 1: "+ label gather", 2: "+ gather + 2 match_any", 3: "pipelined idx, gather lead 1", 4: "pipelined, gather lead 2", 6: "pipelined, gather lead 4", 7: "chunk-pipelined lead 1", 8: "first 64 entries only (bound)", 9: "pipelined + next-chunk L2 prefetch"}
 for mode, name in [(m, NAMES[m]) for m in MODES]:
     for grid, contig in [(g, c) for g, c in ((148 * 4, 0), (148 * 6, 0), (148 * 8, 0), (148 * 4, 1), (148 * 8, 1)) if mode < 3 or g == 148 * 4]:
         ts = []
@@ -139,3 +150,19 @@ for mode, name in [(m, NAMES[m]) for m in MODES]:
             m.run(g.offsets, g.indices, w, labels, rows, out, mode, grid, contig)
             e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
         print(f"{name:28s} grid {grid} contig {contig}: {min(ts):.3f} ms", flush=True)
+
+# sweep-0 schedule in phases: the contiguous-run schedule applied to P
+# consecutive slices of the bin one after another (smaller label window per
+# phase, runs 1/P as long)
+if os.environ.get("SKEL_PHASES"):
+    for mode in (3,):
+        for P in [int(x) for x in os.environ["SKEL_PHASES"].split(",")]:
+            ts = []
+            n = rows.numel()
+            for r in range(3):
+                torch.cuda.synchronize(); e0.record()
+                for p in range(P):
+                    sl = rows[p * n // P:(p + 1) * n // P]
+                    m.run(g.offsets, g.indices, w, labels, sl, out, mode, 148 * 4, 1)
+                e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
+            print(f"{NAMES[mode]:28s} contiguous runs in {P} phases: {min(ts):.3f} ms", flush=True)
