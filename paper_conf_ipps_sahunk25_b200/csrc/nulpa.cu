@@ -184,18 +184,20 @@ __device__ __forceinline__ bool ht_accumulate(int32_t *Hk, float *Hv, const Hash
 
 // Algorithm 2's probe sequence without the value update: find the slot
 // holding k or claim an empty one with atomicCAS (R5 linear continuation).
-__device__ __forceinline__ uint32_t ht_claim(int32_t *Hk, const Hash &h, int32_t k) {
+__device__ __forceinline__ uint32_t ht_claim(int32_t *Hk, const Hash &h, int32_t k, bool *fresh = nullptr) {
     const uint32_t p1 = h.p1;
     uint32_t i = fastmod((uint32_t)k, h.m1, p1);
     uint32_t di = p1 > 1 ? 1u : 0u;
     uint32_t km = fastmod((uint32_t)k, h.m2, h.p2);
     if (km >= p1) km -= p1;
     if (km >= p1) km -= p1;
+    if (fresh) *fresh = false;
     for (int t = 0; t < kMaxRetries; ++t) {
         int32_t cur = *((volatile int32_t *)&Hk[i]);
         if (cur == k) return i;
         if (cur == kEmpty) {
             int32_t old = atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty && fresh) *fresh = true;
             if (old == kEmpty || old == k) return i;
         }
         i += di;
@@ -209,6 +211,7 @@ __device__ __forceinline__ uint32_t ht_claim(int32_t *Hk, const Hash &h, int32_t
         if (cur == k) return i;
         if (cur == kEmpty) {
             int32_t old = atomicCAS(&Hk[i], kEmpty, k);
+            if (old == kEmpty && fresh) *fresh = true;
             if (old == kEmpty || old == k) return i;
         }
         i = i + 1 == p1 ? 0 : i + 1;
@@ -653,6 +656,9 @@ constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 // order, and every re-reading lane stored to that address itself.
 #ifndef NULPA_WARP_SYNC
 #define NULPA_WARP_SYNC 1
+#endif
+#ifndef NULPA_BLOCK_LIST
+#define NULPA_BLOCK_LIST 1               // k_block: list the claimed slots; scan and reset only those
 #endif
 #ifndef NULPA_EPOCH
 #define NULPA_EPOCH 1                    // 0: zero the k_warp table before every vertex
@@ -1312,7 +1318,13 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
     int32_t *Hk = reinterpret_cast<int32_t *>(dyn_b);                 // keys (kEmpty = free)
     uint32_t *Hc = reinterpret_cast<uint32_t *>(Hk + cap);            // unit-weight counts
     float *Hf = reinterpret_cast<float *>(Hc + cap);                  // other weights
+#if NULPA_BLOCK_LIST
+    uint32_t *Hlist = reinterpret_cast<uint32_t *>(Hf + cap);         // slots claimed by this vertex
+    int32_t *rowi = reinterpret_cast<int32_t *>(Hlist + cap);         // 2 index buffers of rowcap
+    __shared__ uint32_t s_nlist;
+#else
     int32_t *rowi = reinterpret_cast<int32_t *>(Hf + cap);            // 2 index buffers of rowcap
+#endif
     float *roww = reinterpret_cast<float *>(rowi + 2 * rowcap);       // 2 weight buffers (W)
     __shared__ __align__(8) uint64_t s_bar[2];
     __shared__ uint64_t s_best[NT / 32];
@@ -1337,6 +1349,16 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
         mbar_init(bar0 + 8, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+#if NULPA_BLOCK_LIST
+    // the table is cleared once; afterwards every vertex resets the slots it
+    // claimed (listed in Hlist) while it scans them for hashtableMaxKey
+    for (int q = threadIdx.x; q < cap; q += NT) {
+        Hk[q] = kEmpty;
+        Hc[q] = 0;
+        Hf[q] = 0.0f;
+    }
+    if (threadIdx.x == 0) s_nlist = 0;
+#endif
     __syncthreads();
     if (threadIdx.x == 0 && (int64_t)blockIdx.x < n) stage(recs[blockIdx.x], 0);
     int i = 0;
@@ -1352,11 +1374,13 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
         const int64_t v = rc.r + a.row_begin;
         Hash h;
         h.init(deg);
+#if !NULPA_BLOCK_LIST
         for (uint32_t q = threadIdx.x; q < h.p1; q += NT) {   // hashtableClear
             Hk[q] = kEmpty;
             Hc[q] = 0;
             Hf[q] = 0.0f;
         }
+#endif
         mbar_wait(bar0 + 8u * b, (uint32_t)(i >> 1) & 1u);
         const int32_t *ri = rowi + b * rowcap + (r_o(rc) & 3);
         const float *rw = roww + b * rowcap + (r_o(rc) & 3);
@@ -1386,15 +1410,40 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
                 const unsigned maxn = __reduce_max_sync(0xFFFFFFFFu, key[u] != kEmpty ? (unsigned)__popc(grp) : 1u);
                 x = maxn > 1 ? group_sum(grp, w[u], maxn) : w[u];
             }
+            uint32_t slot = 0;
+            bool fresh = false;
             if (leader) {
-                const uint32_t slot = ht_claim(Hk, h, key[u]);
+                slot = ht_claim(Hk, h, key[u], &fresh);
                 if (eq) atomicAdd(&Hc[slot], (uint32_t)__popc(grp));
                 else atomicAdd(&Hf[slot], x);
             }
+#if NULPA_BLOCK_LIST
+            // list the newly claimed slots: one shared atomic per warp and batch
+            const unsigned fm = __ballot_sync(0xFFFFFFFFu, fresh);
+            if (fm) {
+                uint32_t base = 0;
+                if (lane == __ffs(fm) - 1) base = atomicAdd(&s_nlist, (uint32_t)__popc(fm));
+                base = __shfl_sync(0xFFFFFFFFu, base, __ffs(fm) - 1);
+                if (fresh) Hlist[base + __popc(fm & ((1u << lane) - 1))] = slot;
+            }
+#endif
         }
         __syncthreads();                                             // table complete
         // hashtableMaxKey: (total, smallest label) as one 64-bit max
         uint64_t best = 0;
+#if NULPA_BLOCK_LIST
+        const uint32_t nl = s_nlist;
+        for (uint32_t q = threadIdx.x; q < nl; q += NT) {
+            const uint32_t sl = Hlist[q];
+            const int32_t kk = Hk[sl];
+            const float t = __fadd_rn((float)Hc[sl], Hf[sl]);
+            const uint64_t c = ((uint64_t)(__float_as_uint(t) + 1) << 32) | (uint32_t)~kk;
+            best = c > best ? c : best;
+            Hk[sl] = kEmpty;                                         // hashtableClear of the claimed slots
+            Hc[sl] = 0;
+            Hf[sl] = 0.0f;
+        }
+#else
         for (uint32_t q = threadIdx.x; q < h.p1; q += NT) {
             const int32_t kk = Hk[q];
             if (kk == kEmpty) continue;
@@ -1402,6 +1451,7 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
             const uint64_t c = ((uint64_t)(__float_as_uint(t) + 1) << 32) | (uint32_t)~kk;
             best = c > best ? c : best;
         }
+#endif
         best = warp_max_u64(best);
         if (lane == 0) s_best[wid] = best;
         __syncthreads();
@@ -1412,6 +1462,9 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
             const int ch = accept_move(cs, rc.ci, sweep_pl(a));
             if (ch) a.lab_out[v] = cs;
             s_changed = ch;
+#if NULPA_BLOCK_LIST
+            s_nlist = 0;                                             // the next vertex's claims come after two more barriers
+#endif
             n_changed += ch;
             n_changed_edges += ch ? deg : 0;
         }
@@ -2480,7 +2533,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             auto launch_block = [&](auto kern, int nt, int maxdeg, const VRec *recs_b, unsigned long long *cnt) -> int {
                 const int cap = (int)capacity_p1((uint32_t)maxdeg) + 1;
                 const int rowcap = (maxdeg + 4 + 3) & ~3;
-                const size_t smem = (size_t)cap * 12 + (size_t)rowcap * 4 * 2 * (W ? 2 : 1);
+                const size_t smem = (size_t)cap * (NULPA_BLOCK_LIST ? 16 : 12) + (size_t)rowcap * 4 * 2 * (W ? 2 : 1);
                 CU(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
                 int per_sm = 0;
                 CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, nt, smem));

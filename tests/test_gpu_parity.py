@@ -212,8 +212,8 @@ def test_compacted_thread_bin_sweep(gname, weighted):
     """The asynchronous bulk thread bin of degree <= 8 (road, k-mer) runs as
     k_tscan + k_tact over a compacted frontier (nulpa.cu).  From a random
     mid-run state (30% of the vertices unprocessed): exactly the unprocessed
-    vertices are processed (Algorithm 1) and no other label
-    moves; every moved label is an own/neighbour label; afterwards a vertex
+    vertices are processed (Algorithm 1; isolated vertices are
+    in no bin and keep label and flag, R7) and no other label moves; every moved label is an own/neighbour label; afterwards a vertex
     is unprocessed iff one of its neighbours moved (line 348: processed
     vertices are cleared first, then marked); dN counts the moves."""
     # large enough for one k_tscan/k_tact launch per sweep (bins spanning
@@ -235,16 +235,18 @@ def test_compacted_thread_bin_sweep(gname, weighted):
     dn = gg.sweep(False, mode=nl.ASYNC)
     C1 = gg.labels(device=False).numpy()
     U1 = gg.flags(device=False).numpy()
-    assert gg.stats()["vertices_processed"][0] - before == int(U0.sum())
+    deg = np.diff(h.offsets)
+    assert gg.stats()["vertices_processed"][0] - before == int(((U0 == 1) & (deg > 0)).sum())   # R7: no bin for degree 0
     moved = C1 != C0
     assert dn == int(moved.sum())
     assert not (moved & (U0 == 0)).any(), "a vertex that was not unprocessed moved"
-    src = np.repeat(np.arange(g.N), np.diff(h.offsets))
+    src = np.repeat(np.arange(g.N), deg)
     j = h.indices
     ok = (src != j) & ((C0[j] == C1[src]) | (C1[j] == C1[src]))       # an own/neighbour label
     assert (np.bincount(src[ok], minlength=g.N)[moved] > 0).all(), "a vertex took a label no neighbour had"
     marked = np.zeros(g.N, dtype=bool)
     marked[h.indices[moved[src]]] = True
+    marked |= (U0 == 1) & (deg == 0)                                    # never processed, flag kept
     assert np.array_equal(U1.astype(bool), marked)
 
 
