@@ -96,8 +96,11 @@ typedef struct nulpa_params {
                                     then ONE CUDA graph whose conditional while node runs sweeps
                                     1.. and Algorithm 1's stop test on the device
                                     -- no host synchronisation per iteration; the graph is built
-                                    once per handle and parameter set.  0 (or timing == 1): the
-                                    host loop, one synchronisation per iteration               */
+                                    once per handle and parameter set, from the handle's second
+                                    nulpa_run on (the first run of a handle takes the host loop:
+                                    building a graph costs more than one run of a small graph
+                                    saves).  0 (or timing == 1): the host loop, one
+                                    synchronisation per iteration                              */
 } nulpa_params;
 
 #define NULPA_TIE_SMALLEST 0
