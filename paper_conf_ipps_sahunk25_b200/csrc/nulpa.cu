@@ -660,6 +660,9 @@ constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 #ifndef NULPA_BLOCK_LIST
 #define NULPA_BLOCK_LIST 1               // k_block: list the claimed slots; scan and reset only those
 #endif
+#ifndef NULPA_MAJORITY
+#define NULPA_MAJORITY 1                 // k_warp: strict-majority shortcut for the vertex's own label (not the first sweep)
+#endif
 #ifndef NULPA_EPOCH
 #define NULPA_EPOCH 1                    // 0: zero the k_warp table before every vertex
 #endif
@@ -1016,8 +1019,8 @@ struct GroupFetcher {
 // are loaded here.  Returns hashtableMaxKey (kEmpty if no neighbour).
 template <bool W, int SLOTS, bool O32>
 __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, int lane, unsigned lanes_below,
-                                             uint64_t row_o, uint32_t dk, int32_t vk, int32_t k0a, int32_t k0b,
-                                             float w0a, float w0b, uint32_t &ep) {
+                                             uint64_t row_o, uint32_t dk, int32_t vk, int32_t ci, int32_t k0a,
+                                             int32_t k0b, float w0a, float w0b, uint32_t &ep) {
     constexpr int U = WarpCfg<SLOTS>::unroll;
     (void)U;
     const int32_t *__restrict__ lab_in = a.lab_in;
@@ -1035,12 +1038,48 @@ __device__ __forceinline__ int32_t warp_fold(const SweepArgs &a, uint32_t tab, i
         return maxn > 1 ? group_sum(grp, w, maxn) : w;
     };
     if (dk <= 32) {
+#if NULPA_MAJORITY
+        if (!a.first && eqw && 2 * __popc(__ballot_sync(0xFFFFFFFFu, k0a == ci)) > __popc(__ballot_sync(0xFFFFFFFFu, k0a != kEmpty)))
+            return ci;                                     // strict majority of the own label (below)
+#endif
         const unsigned grp = __match_any_sync(0xFFFFFFFFu, k0a);
         const bool leader = k0a != kEmpty && (grp & lanes_below) == 0;
         const float x = group_total(grp, k0a, w0a, eqw);
         bw = leader ? __float_as_uint(x) + 1 : 0u;
         bk = k0a;
     } else {
+#if NULPA_MAJORITY
+        // Past the first sweep most neighbourhoods hold one label.  If the
+        // vertex's own label C[i] has a strict majority of its (unit)
+        // neighbour weights, it is hashtableMaxKey -- no other label can
+        // reach its total, so no tie either -- and the vertex does not move:
+        // the same decision as the table fold, for two ballots per batch.
+        if (!a.first && eqw) {
+            uint32_t own = __popc(__ballot_sync(0xFFFFFFFFu, k0a == ci)) + __popc(__ballot_sync(0xFFFFFFFFu, k0b == ci));
+            uint32_t tot = __popc(__ballot_sync(0xFFFFFFFFu, k0a != kEmpty)) + __popc(__ballot_sync(0xFFFFFFFFu, k0b != kEmpty));
+            if (2 * own > tot) {
+                // rows past 64 entries: a majority in the first 64 -- count the
+                // rest (two batches of loads in flight per step); on failure the
+                // table fold below re-reads them
+                bool unit = true;
+                const uint64_t el = at(row_o, (uint32_t)lane);
+                for (uint32_t b = 64; b < dk && unit; b += 64) {
+                    const bool oka = b + lane < dk, okb = b + 32 + lane < dk;
+                    const int32_t ja = oka ? ld_stream(a.indices + el + b) : -1;
+                    const int32_t jb = okb ? ld_stream(a.indices + el + b + 32) : -1;
+                    float xa = 1.0f, xb = 1.0f;
+                    if (W && oka) xa = ld_stream(a.weights + el + b);
+                    if (W && okb) xb = ld_stream(a.weights + el + b + 32);
+                    const int32_t ka = (ja >= 0 && ja != vk) ? ld_label(lab_in + ja) : kEmpty;
+                    const int32_t kb = (jb >= 0 && jb != vk) ? ld_label(lab_in + jb) : kEmpty;
+                    if (W) unit = __all_sync(0xFFFFFFFFu, (ka == kEmpty || xa == 1.0f) && (kb == kEmpty || xb == 1.0f));
+                    own += __popc(__ballot_sync(0xFFFFFFFFu, ka == ci)) + __popc(__ballot_sync(0xFFFFFFFFu, kb == ci));
+                    tot += __popc(__ballot_sync(0xFFFFFFFFu, ka != kEmpty)) + __popc(__ballot_sync(0xFFFFFFFFu, kb != kEmpty));
+                }
+                if (unit && 2 * own > tot) return ci;
+            }
+        }
+#endif
         auto table_row = [&](auto cap) {
             constexpr uint32_t P = decltype(cap)::value;
             // hashtableClear: next epoch; zero the whole table when the epoch wraps
@@ -1239,7 +1278,7 @@ __global__ void __launch_bounds__(WarpCfg<SLOTS>::warps * 32, WarpCfg<SLOTS>::ct
         }
         // ---- fold vertex n ----
         const int32_t vk = rc.r + (int32_t)a.row_begin;
-        const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, k0a, k0b, w0a, w0b, ep);
+        const int32_t cs = warp_fold<W, SLOTS, O32>(a, tab, lane, lanes_below, r_o(rc), dk, vk, rc.ci, k0a, k0b, w0a, w0b, ep);
         if (accept_move(cs, rc.ci, pl)) {
             c_ch += 1;
             c_che += dk;
@@ -1329,6 +1368,9 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
     __shared__ __align__(8) uint64_t s_bar[2];
     __shared__ uint64_t s_best[NT / 32];
     __shared__ int s_changed;
+#if NULPA_MAJORITY
+    __shared__ uint32_t s_maj[3];            // own-label count, neighbour count, non-unit weight seen
+#endif
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(&s_bar[0]);
     const int64_t n = (int64_t)*count;
@@ -1349,6 +1391,9 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
         mbar_init(bar0 + 8, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+#if NULPA_MAJORITY
+    if (threadIdx.x < 3) s_maj[threadIdx.x] = 0;
+#endif
 #if NULPA_BLOCK_LIST
     // the table is cleared once; afterwards every vertex resets the slots it
     // claimed (listed in Hlist) while it scans them for hashtableMaxKey
@@ -1398,9 +1443,36 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
                 if (W) w[u] = rw[e];
             }
         }
+#if NULPA_MAJORITY
+        // strict majority of the vertex's own label (unit weights, past the
+        // first sweep): it is hashtableMaxKey and the vertex does not move --
+        // no table work (see warp_fold)
+        if (!a.first) {
+            uint32_t own = 0, tot = 0;
+            bool unit = true;
+#pragma unroll
+            for (int u = 0; u < R; ++u) {
+                if ((uint32_t)(u * NT) + (uint32_t)(wid * 32) >= deg) break;   // warp-uniform
+                own += __popc(__ballot_sync(0xFFFFFFFFu, key[u] == rc.ci));
+                tot += __popc(__ballot_sync(0xFFFFFFFFu, key[u] != kEmpty));
+                if (W) unit = unit && __all_sync(0xFFFFFFFFu, key[u] == kEmpty || w[u] == 1.0f);
+            }
+            if (lane == 0 && tot) {
+                atomicAdd(&s_maj[0], own);
+                atomicAdd(&s_maj[1], tot);
+                if (!unit) s_maj[2] = 1;
+            }
+        }
+#endif
         __syncthreads();                                             // table cleared
+#if NULPA_MAJORITY
+        const bool maj = !a.first && s_maj[2] == 0 && 2 * s_maj[0] > s_maj[1];
+#else
+        constexpr bool maj = false;
+#endif
 #pragma unroll
         for (int u = 0; u < R; ++u) {
+            if (maj) break;
             if ((uint32_t)(u * NT) + (uint32_t)(wid * 32) >= deg) break;   // warp-uniform
             const unsigned grp = __match_any_sync(0xFFFFFFFFu, key[u]);
             const bool leader = key[u] != kEmpty && (grp & ((1u << lane) - 1)) == 0;
@@ -1458,12 +1530,15 @@ __global__ void __launch_bounds__(NT) k_block(SweepArgs a, const VRec *__restric
         if (threadIdx.x == 0) {
             uint64_t bb = 0;
             for (int q = 0; q < NT / 32; ++q) bb = s_best[q] > bb ? s_best[q] : bb;
-            const int32_t cs = bb ? (int32_t)~(uint32_t)bb : kEmpty;
+            const int32_t cs = maj ? rc.ci : bb ? (int32_t)~(uint32_t)bb : kEmpty;
             const int ch = accept_move(cs, rc.ci, sweep_pl(a));
             if (ch) a.lab_out[v] = cs;
             s_changed = ch;
 #if NULPA_BLOCK_LIST
             s_nlist = 0;                                             // the next vertex's claims come after two more barriers
+#endif
+#if NULPA_MAJORITY
+            s_maj[0] = s_maj[1] = s_maj[2] = 0;                      // likewise the next vertex's counts
 #endif
             n_changed += ch;
             n_changed_edges += ch ? deg : 0;
