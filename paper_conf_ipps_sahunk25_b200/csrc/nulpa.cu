@@ -1581,6 +1581,7 @@ struct GiantArgs {
     uint8_t *active;             // [ng]
     uint8_t *changed;            // [ng]
     unsigned long long *best;    // [ng] packed (weight, tie rank) maximum
+    unsigned long long *maj;     // [3 ng] own-label count, neighbour count, non-unit weights seen (majority shortcut)
 };
 
 template <bool SYNC>
@@ -1593,7 +1594,58 @@ __global__ void k_giant_snapshot(SweepArgs a, GiantArgs g, int64_t ng) {
     g.changed[k] = 0;
     g.best[k] = 0;
     g.occ_n[k] = 0;
+    g.maj[3 * k] = g.maj[3 * k + 1] = g.maj[3 * k + 2] = 0;
     if (!SYNC && f) a.flag_in[v] = 0;
+}
+
+#if NULPA_MAJORITY
+// Majority shortcut for giant vertices (every sweep but the first after a
+// reset): one pass over the active giants' rows counting the neighbours that
+// hold the vertex's own label, the neighbours, and non-unit weights; a giant
+// whose own label holds a strict majority (unit weights) skips the table
+// fold and keeps its label (k_giant_accumulate / k_giant_decide).
+template <bool W>
+__global__ void __launch_bounds__(kBlockThreads) k_giant_count(SweepArgs a, GiantArgs g) {
+    const int64_t c = blockIdx.x;
+    const int32_t gi = g.chunk_g[c];
+    if (!g.active[gi]) return;
+    const int64_t v = g.verts[gi] + a.row_begin;
+    const int32_t ci = a.lab_in[v];
+    const int64_t e0 = g.chunk_e0[c], e1 = g.chunk_e1[c];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    uint32_t own = 0, tot = 0, nonunit = 0;
+    for (int64_t b = e0 + wid * 32; b < e1; b += 2 * kBlockThreads) {
+        int32_t j[2] = {-1, -1};
+        float w[2] = {1.0f, 1.0f};
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const int64_t e = b + u * kBlockThreads + lane;
+            if (e < e1) {
+                j[u] = ld_stream(a.indices + e);
+                if (W) w[u] = ld_stream(a.weights + e);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const int32_t key = (j[u] >= 0 && j[u] != (int32_t)v) ? a.lab_in[j[u]] : kEmpty;
+            own += __popc(__ballot_sync(0xFFFFFFFFu, key == ci));
+            tot += __popc(__ballot_sync(0xFFFFFFFFu, key != kEmpty));
+            if (W) nonunit += __popc(__ballot_sync(0xFFFFFFFFu, key != kEmpty && w[u] != 1.0f));
+        }
+    }
+    if (lane == 0 && tot) {
+        atomicAdd(&g.maj[3 * gi], (unsigned long long)own);
+        atomicAdd(&g.maj[3 * gi + 1], (unsigned long long)tot);
+        if (nonunit) atomicAdd(&g.maj[3 * gi + 2], (unsigned long long)nonunit);
+    }
+}
+#endif
+__device__ __forceinline__ bool giant_majority(const SweepArgs &a, const GiantArgs &g, int64_t gi) {
+#if NULPA_MAJORITY
+    return !a.first && g.maj[3 * gi + 2] == 0 && 2 * g.maj[3 * gi] > g.maj[3 * gi + 1];
+#else
+    return false;
+#endif
 }
 
 template <bool SYNC, bool W>
@@ -1610,6 +1662,10 @@ __global__ void __launch_bounds__(kBlockThreads) k_giant_accumulate(SweepArgs a,
     const int32_t r = g.verts[gi];
     const int64_t v = r + a.row_begin;
     const int64_t e0 = g.chunk_e0[c], e1 = g.chunk_e1[c];
+    if (giant_majority(a, g, gi)) {                        // no table fold (k_giant_count)
+        if (threadIdx.x == 0) atomicAdd(&a.ctr[5 + 3], (unsigned long long)(e1 - e0));
+        return;
+    }
     for (int s = threadIdx.x; s < kGiantCap; s += kBlockThreads) {
         Hk[s] = kEmpty;
         Hv[s] = 0.0f;
@@ -1702,7 +1758,7 @@ __global__ void k_giant_decide(SweepArgs a, GiantArgs g, int64_t ng) {
     TieOrder to;
     to.init(h);
     const unsigned long long b = g.best[gi];
-    const int32_t cs = b ? cand_label(b, to) : kEmpty;
+    const int32_t cs = giant_majority(a, g, gi) ? a.lab_in[v] : b ? cand_label(b, to) : kEmpty;
     const bool ch = accept_move(cs, a.lab_in[v], sweep_pl(a));
     if (ch) {
         a.lab_out[v] = cs;
@@ -2104,6 +2160,7 @@ struct nulpa_graph {
     float *gvals = nullptr;
     uint8_t *gactive = nullptr, *gchanged = nullptr;
     unsigned long long *gbest = nullptr;
+    unsigned long long *gmaj = nullptr;      // [3 ng] majority-shortcut counts of the giant bin
     // counters
     unsigned long long *ctr = nullptr;       // device [kMaxIter+1][kCtr]
     unsigned long long *ctr_host = nullptr;  // pinned
@@ -2218,6 +2275,8 @@ void free_bins(nulpa_graph *g) {
     dfree(g->gchanged);
     dfree(g->gbest);
     g->gbest = nullptr;
+    dfree(g->gmaj);
+    g->gmaj = nullptr;
     g->chunk_g = nullptr;
     g->chunk_e0 = g->chunk_e1 = g->table_off = nullptr;
     g->gkeys = g->occ = g->occ_n = nullptr;
@@ -2408,6 +2467,7 @@ int build_bins(nulpa_graph *g, int32_t t1, int32_t t2, int32_t t3) {
         CHECK(dalloc(&g->gactive, (size_t)ng));
         CHECK(dalloc(&g->gchanged, (size_t)ng));
         CHECK(dalloc(&g->gbest, (size_t)ng));
+        CHECK(dalloc(&g->gmaj, (size_t)(3 * ng)));
         // on the handle's stream (every bin kernel is ordered after the
         // cudaStreamSynchronize(g->stream) below; the host vectors outlive it)
         CU(cudaMemcpyAsync(g->chunk_g, cg.data(), cg.size() * sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
@@ -2585,10 +2645,17 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
             ga.active = g->gactive;
             ga.changed = g->gchanged;
             ga.best = g->gbest;
+            ga.maj = g->gmaj;
             const size_t smem = kGiantCap * (sizeof(int32_t) + sizeof(float)) + kGiantChunk * sizeof(uint16_t);
             // set on every launch: the attribute is per device, the handle may live on any
             CU(cudaFuncSetAttribute(k_giant_accumulate<SYNC, W>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             k_giant_snapshot<SYNC><<<grid_for(ng, 256), 256, 0, cs>>>(a, ga, ng);
+#if NULPA_MAJORITY
+            if (!a.first) {
+                k_giant_count<W><<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
+                g->stats.launches[3] += 1;
+            }
+#endif
             k_giant_accumulate<SYNC, W><<<(unsigned)g->n_chunks, kBlockThreads, smem, cs>>>(a, ga);
             k_giant_decide<SYNC><<<grid_for(ng, 128), 128, 0, cs>>>(a, ga, ng);
             k_giant_finish<<<(unsigned)g->n_chunks, kBlockThreads, 0, cs>>>(a, ga);
