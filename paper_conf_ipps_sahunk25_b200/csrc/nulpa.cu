@@ -3,7 +3,7 @@
 //
 // Paper: PAPER.md (Sahu, nu-LPA).  Algorithm 1 is the
 // sweep/loop structure, Algorithm 2 the per-vertex
-// hashtable, Eq. 1 the modularity.  Readings R1..R12 are
+// hashtable, Eq. 1 the modularity.  Readings R1..R13 are
 // listed in DESIGN.md.  This file shares no code with oracle/.
 //
 // Layout in HBM:
@@ -15,13 +15,20 @@
 //
 // Kernels of one sweep (lpaMove): thread bin, then the warp bin on a
 // high-priority stream with block + giant on a low-priority stream filling its
-// tail (bin_order 3, default; bin_order 1 = thread -> warp -> block -> giant
-// in order on the handle's stream, hubs last):
-//   k_giant_snapshot / k_giant_accumulate / k_giant_decide / k_giant_finish
-//   k_block   one CTA per vertex, shared-memory table (<= 4095 slots)
-//   k_frontier + k_warp   compacted frontier; one warp per vertex, pipelined,
-//                         shared-memory table (<= 511 slots)
-//   k_thread  one thread per vertex, labels in registers (degree < 32)
+// tail (bin_order 3; bin_order 1 = thread -> warp -> block -> giant in order
+// on the handle's stream, hubs last; bin_order 4, the default, picks 3 when
+// the warp bin holds >= 2/3 of the CSR entries, else 1):
+//   k_giant_snapshot / [k_giant_count] / k_giant_accumulate / k_giant_decide / k_giant_finish
+//             chunked CTAs per vertex, global-memory tables
+//   k_frontier + k_block   one CTA per vertex (4 or 8 warps), TMA row staging,
+//                          shared-memory table (<= 2047 slots)
+//   k_frontier + k_warp    compacted frontier; one warp per vertex, pipelined,
+//                          epoch-tagged shared-memory table (<= 511 slots)
+//   k_thread  one thread per vertex, labels in registers (degree < 16), or
+//   k_tscan + k_tact       the same over a compacted frontier (asynchronous
+//                          bulk bins of degree <= 8: road, k-mer)
+// Past the first sweep, a vertex whose own label holds a strict majority of
+// its (unit) neighbour weights skips the table fold (the majority shortcut).
 
 #include "nulpa.h"
 
