@@ -2554,7 +2554,7 @@ static_assert(kThreadWaves <= kCtr - kCtrTScan, "one compaction counter per wave
 #define NULPA_TCOMPACT 1                 // asynchronous bulk thread bins: compacted frontier
 #endif
 template <bool SYNC, bool W>
-int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
+int launch_thread_bin(nulpa_graph *g, const SweepArgs &a, cudaStream_t st) {
     const int64_t n = g->bin_n[0];
     const int64_t md = g->bin_maxdeg[0];     // register table sized by the bin's largest degree
     // a bin spanning >= kThreadWaves grid-stride steps is already swept in
@@ -2578,22 +2578,22 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a) {
                               : grid_for(m, kThreadThreads, num_sms() * 32);
         if (compact) {
             unsigned long long *cnt = a.ctr + kCtrTScan + w;
-            k_tscan<<<grid_for(m, 4 * kTScanThreads, num_sms() * 8), kTScanThreads, 0, g->stream>>>(a, list, m, g->trows, cnt);
+            k_tscan<<<grid_for(m, 4 * kTScanThreads, num_sms() * 8), kTScanThreads, 0, st>>>(a, list, m, g->trows, cnt);
             if (md <= 4)
-                k_tact<W, 4, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, g->trows, cnt);
+                k_tact<W, 4, 4><<<grid, kThreadThreads, 0, st>>>(a, g->trows, cnt);
             else
-                k_tact<W, 8, 2><<<grid, kThreadThreads, 0, g->stream>>>(a, g->trows, cnt);
+                k_tact<W, 8, 2><<<grid, kThreadThreads, 0, st>>>(a, g->trows, cnt);
             CU(cudaGetLastError());
             continue;
         }
         if (md <= 4)
-            k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+            k_thread<SYNC, W, 4><<<grid, kThreadThreads, 0, st>>>(a, list, m, bulk);
         else if (md <= 8)
-            k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+            k_thread<SYNC, W, 8><<<grid, kThreadThreads, 0, st>>>(a, list, m, bulk);
         else if (md <= 16)
-            k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+            k_thread<SYNC, W, 16><<<grid, kThreadThreads, 0, st>>>(a, list, m, bulk);
         else
-            k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, g->stream>>>(a, list, m, bulk);
+            k_thread<SYNC, W, 32><<<grid, kThreadThreads, 0, st>>>(a, list, m, bulk);
         CU(cudaGetLastError());
     }
     g->stats.launches[0] += (int)waves * (compact ? 2 : 1) - 1;
@@ -2764,7 +2764,7 @@ int sweep_impl(nulpa_graph *g, int pickless, const nulpa_params &p, unsigned lon
         const int64_t n = g->bin_n[0];
         CHECK(rec(0, 0));
         if (n > 0) {
-            CHECK((launch_thread_bin<SYNC, W>(g, a)));
+            CHECK((launch_thread_bin<SYNC, W>(g, a, cs)));
             g->stats.launches[0] += 1;
         }
         CHECK(rec(0, 1));
