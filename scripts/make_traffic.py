@@ -37,12 +37,22 @@ def dram(k):
 
 ids = sorted(per, key=int)
 if binname == "warp":
-    main = [k for k in ids if "k_warp" in name[k] and ", 512" in name[k]]
-    front = [ids[ids.index(k) - 1] for k in main]
-    assert all("k_frontier" in name[f] for f in front), [name[f] for f in front]
-    b = [dram(f) + dram(w) for f, w in zip(front, main)]
-    kernels = ["k_frontier", "k_warp"]
-    extra = {"k_warp_per_launch": [dram(w) for w in main], "k_frontier_per_launch": [dram(f) for f in front]}
+    # per sweep: the warp-bin k_frontier, k_warp_easy (two-pass sweeps) and k_warp
+    main = [k for k in ids if "k_warp<" in name[k] and ", 512" in name[k]]
+    front, easy = [], []
+    for k in main:
+        j = ids.index(k) - 1
+        e = None
+        if "k_warp_easy" in name[ids[j]]:
+            e = ids[j]
+            j -= 1
+        assert "k_frontier" in name[ids[j]], name[ids[j]]
+        front.append(ids[j])
+        easy.append(e)
+    b = [dram(f) + dram(w) + (dram(e) if e else 0.0) for f, w, e in zip(front, main, easy)]
+    kernels = ["k_frontier", "k_warp_easy", "k_warp"] if any(easy) else ["k_frontier", "k_warp"]
+    extra = {"k_warp_per_launch": [dram(w) for w in main], "k_frontier_per_launch": [dram(f) for f in front],
+             "k_warp_easy_per_launch": [dram(e) if e else 0.0 for e in easy]}
 elif binname == "block":
     # per sweep: the block-bin k_frontier (the one right before a k_block launch) and the k_block
     # launches that follow it (4-warp TMA k_block below wide_degree, 8-warp above)
