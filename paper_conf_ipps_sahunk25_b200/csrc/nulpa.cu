@@ -447,7 +447,7 @@ __global__ void __launch_bounds__(kThreadThreads) k_thread(SweepArgs a, const in
 // i as processed"); one global atomic per tile.  k_tact then gives every
 // thread 4 consecutive compacted rows (the ID-order propagation of the
 // grid-stride k_thread: vertex u sees the labels rows u-1.. of its quad
-// wrote) and issues the loads of V of them at once -- offsets, indices,
+// wrote) and issues the loads of all 4 of them at once -- offsets, indices,
 // weights, neighbour labels -- before deciding them in order; a label
 // gathered before an earlier row of the quad moved is patched to the new
 // label (as k_warp does for its pipelined vertex).  Late sweeps of a road
@@ -507,8 +507,8 @@ __global__ void __launch_bounds__(kTScanThreads) k_tscan(SweepArgs a, const int3
     }
 }
 
-// V rows of a quad have their loads in flight together (V = 4 for degrees
-// <= 4: road; 2 above)
+// V rows of a quad have their loads in flight together (V = 4: road, and
+// k-mer at MAXD 8 with NULPA_TACT_V8)
 template <bool W, int MAXD, int V>
 __global__ void __launch_bounds__(kThreadThreads) k_tact(SweepArgs a, const int32_t *__restrict__ rows,
                                                          const unsigned long long *__restrict__ count) {
@@ -2550,6 +2550,9 @@ int ensure_bins(nulpa_graph *g, const nulpa_params &p) {
 #endif
 constexpr int kThreadWaves = NULPA_THREAD_WAVES;
 static_assert(kThreadWaves <= kCtr - kCtrTScan, "one compaction counter per wave");
+#ifndef NULPA_TACT_V8
+#define NULPA_TACT_V8 4                  // k_tact rows in flight together for degrees 5..8 (k-mer 3.93e9 edges/s; 2 rows: 3.79e9)
+#endif
 #ifndef NULPA_TCOMPACT
 #define NULPA_TCOMPACT 1                 // asynchronous bulk thread bins: compacted frontier
 #endif
@@ -2582,7 +2585,7 @@ int launch_thread_bin(nulpa_graph *g, const SweepArgs &a, cudaStream_t st) {
             if (md <= 4)
                 k_tact<W, 4, 4><<<grid, kThreadThreads, 0, st>>>(a, g->trows, cnt);
             else
-                k_tact<W, 8, 2><<<grid, kThreadThreads, 0, st>>>(a, g->trows, cnt);
+                k_tact<W, 8, NULPA_TACT_V8><<<grid, kThreadThreads, 0, st>>>(a, g->trows, cnt);
             CU(cudaGetLastError());
             continue;
         }
