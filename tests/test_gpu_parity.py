@@ -109,6 +109,40 @@ def test_sync_sweep_from_random_state(gname, pickless):
         np.testing.assert_array_equal(gg.flags(device=False).numpy(), U1)
 
 
+@pytest.mark.parametrize("gname", ["sbm", "web", "hub", "rmat", "cliques"])
+def test_sync_sweep_majority_states(gname):
+    """The majority shortcut (past the first sweep after a reset, a vertex
+    whose own label holds a strict majority of its unit-weight neighbours
+    keeps it without a table fold -- k_warp, k_block, the giant bin) equals
+    the table fold: from a near-converged state (the oracle's synchronous
+    result with 10% of the labels moved to a random neighbour's label, every
+    vertex unprocessed), one synchronous sweep is bit-exact with the oracle
+    under every bin configuration; most vertices take the shortcut."""
+    g = GRAPHS[gname](False)
+    h = host(g)
+    C, _, _ = oracle.lpa(h, sync=True)
+    rng = np.random.default_rng(13)
+    deg = np.diff(h.offsets)
+    C0 = C.astype(np.int32).copy()
+    for i in np.nonzero((rng.random(g.N) < 0.1) & (deg > 0))[0]:
+        C0[i] = C[h.indices[h.offsets[i] + rng.integers(deg[i])]]
+    U0 = np.ones(g.N, dtype=np.uint8)
+    src = np.repeat(np.arange(g.N), deg)
+    nb = src != h.indices
+    own = np.bincount(src[nb & (C0[h.indices] == C0[src])], minlength=g.N)
+    tot = np.bincount(src[nb], minlength=g.N)
+    assert (2 * own > tot).mean() > 0.5                     # the shortcut is the common case
+    dn, C1, U1, _, _ = oracle.lpa_move_sync(h, C0, U0, False)
+    gg = to_gpu(g)
+    gg.sweep(False, mode=nl.SYNC)                            # past the first sweep after create
+    for bins in BINS.values():
+        gg.set_labels(torch.from_numpy(C0).cuda(), torch.from_numpy(U0).cuda())
+        got = gg.sweep(False, mode=nl.SYNC, **bins)
+        assert got == dn
+        np.testing.assert_array_equal(gg.labels(device=False).numpy(), C1)
+        np.testing.assert_array_equal(gg.flags(device=False).numpy(), U1)
+
+
 # ---------------------------------------------------------------------------
 # synchronous mode, weighted: label-for-label except float32 near-ties
 # ---------------------------------------------------------------------------
