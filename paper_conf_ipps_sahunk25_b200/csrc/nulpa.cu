@@ -668,7 +668,7 @@ constexpr int kWarpSlots = 512;          // largest class: p1 = 511
 #define NULPA_BLOCK_LIST 1               // k_block: list the claimed slots; scan and reset only those
 #endif
 #ifndef NULPA_MAJORITY
-#define NULPA_MAJORITY 1                 // k_warp: strict-majority shortcut for the vertex's own label (not the first sweep)
+#define NULPA_MAJORITY 1                 // k_warp, k_block, giant bin: strict-majority shortcut for the vertex's own label (not the first sweep)
 #endif
 #ifndef NULPA_EPOCH
 #define NULPA_EPOCH 1                    // 0: zero the k_warp table before every vertex
