@@ -913,7 +913,7 @@ constexpr int kWideSlots = 1024, kWideWarps = 4, kWideCtasPerSm = 6;
 #define NULPA_WIDE_GROUP 4
 #endif
 #ifndef NULPA_T255_MAX
-#define NULPA_T255_MAX 64                // k_warp: 255-slot tables below this degree, 511 above
+#define NULPA_T255_MAX 33                // k_warp: 255-slot tables below this degree, 511 above (33: always 511 -- with epoch tags a bigger table costs no clearing and has fewer collisions: web 72.5 -> 73.9e9 edges/s)
 #endif
 #ifndef NULPA_FIRST_BIG
 #define NULPA_FIRST_BIG 0                // 1: 511-slot tables for every degree in the first sweep
